@@ -1,0 +1,120 @@
+"""CPU oracle for the 2D inclusive summed-area table -- TEST INFRASTRUCTURE.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` leg may import this package.  The product path
+(``paper_conf_cluster_chenwttm18_b200``) never imports it and shares no code
+with it (the seeded input generator ``satgen`` is the only common module).
+
+The arithmetic lives in ``sat_oracle.c`` (see its header for the paper
+passages each function follows); this module is ctypes marshalling only.
+
+Pairs: 0 = 8u->32s (int32 output, wrap mod 2^32), 1 = 32f->32f (fp64 output of
+an fp64 recurrence), 2 = 64f->64f (fp64 output of a double-double recurrence).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+PAIR_8U32S, PAIR_32F32F, PAIR_64F64F = 0, 1, 2
+IN_DTYPE = {PAIR_8U32S: np.uint8, PAIR_32F32F: np.float32, PAIR_64F64F: np.float64}
+OUT_DTYPE = {PAIR_8U32S: np.int32, PAIR_32F32F: np.float64, PAIR_64F64F: np.float64}
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liboracle.so")
+SRC_PATH = os.path.join(_HERE, "sat_oracle.c")
+
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc (plain -O2, no fast-math, no contraction)."""
+    if force or not os.path.exists(LIB_PATH) or os.path.getmtime(LIB_PATH) < os.path.getmtime(SRC_PATH):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math",
+                               "-fPIC", "-shared", "-o", LIB_PATH, SRC_PATH])
+    return LIB_PATH
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(LIB_PATH)
+        i64, vp = ctypes.c_int64, ctypes.c_void_p
+        L.oracle_sat.argtypes = [ctypes.c_int, vp, i64, i64, i64, vp, i64]
+        L.oracle_sat_64f_plain.argtypes = [vp, i64, i64, i64, vp, i64]
+        L.oracle_sat_gen_rows.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_uint64, i64,
+                                          ctypes.c_double, i64, i64, vp, i64, vp]
+        L.oracle_alg1_8u32s.argtypes = [vp, i64, i64, i64, vp, i64]
+        L.oracle_alg1_f64.argtypes = [ctypes.c_int, vp, i64, i64, i64, vp, i64]
+        for f in (L.oracle_sat, L.oracle_sat_64f_plain, L.oracle_sat_gen_rows, L.oracle_alg1_8u32s,
+                  L.oracle_alg1_f64):
+            f.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def pair_of(a: np.ndarray) -> int:
+    return {np.dtype(np.uint8): PAIR_8U32S, np.dtype(np.float32): PAIR_32F32F,
+            np.dtype(np.float64): PAIR_64F64F}[a.dtype]
+
+
+def _check(rc: int, what: str):
+    if rc != 0:
+        raise RuntimeError(f"{what} failed with oracle status {rc}")
+
+
+def sat(A: np.ndarray) -> np.ndarray:
+    """Inclusive SAT of a 2-D host image (row stride may be padded)."""
+    assert A.ndim == 2 and (A.size == 0 or A.strides[1] == A.itemsize)
+    pair = pair_of(A)
+    H, W = A.shape
+    S = np.empty((H, W), dtype=OUT_DTYPE[pair])
+    if A.size == 0:
+        return S
+    _check(lib().oracle_sat(pair, A.ctypes.data, H, W, A.strides[0], S.ctypes.data, S.strides[0]),
+           "oracle_sat")
+    return S
+
+
+def sat_batched(A: np.ndarray) -> np.ndarray:
+    return np.stack([sat(a) for a in A]) if A.ndim == 3 else sat(A)
+
+
+def sat_64f_plain(A: np.ndarray) -> np.ndarray:
+    """Plain fp64 recurrence for 64f input (sanity form; reading R4)."""
+    assert A.dtype == np.float64 and A.ndim == 2 and A.strides[1] == 8
+    H, W = A.shape
+    S = np.empty((H, W), dtype=np.float64)
+    _check(lib().oracle_sat_64f_plain(A.ctypes.data, H, W, A.strides[0], S.ctypes.data,
+                                      S.strides[0]), "oracle_sat_64f_plain")
+    return S
+
+
+def alg1(A: np.ndarray) -> np.ndarray:
+    """Algorithm 1 of the paper."""
+    assert A.ndim == 2 and A.strides[1] == A.itemsize
+    H, W = A.shape
+    pair = pair_of(A)
+    if pair == PAIR_8U32S:
+        J = np.empty((H, W), dtype=np.int32)
+        _check(lib().oracle_alg1_8u32s(A.ctypes.data, H, W, A.strides[0], J.ctypes.data,
+                                       J.strides[0]), "oracle_alg1_8u32s")
+    else:
+        J = np.empty((H, W), dtype=np.float64)
+        _check(lib().oracle_alg1_f64(pair, A.ctypes.data, H, W, A.strides[0], J.ctypes.data,
+                                     J.strides[0]), "oracle_alg1_f64")
+    return J
+
+
+def sat_gen_rows(pair: int, H: int, W: int, rows, seed: int = 0, img: int = 0, mode: int = 0,
+                 value: float = 0.0) -> np.ndarray:
+    """Selected rows of the SAT of the satgen image (seed, img); O(W) memory."""
+    rows = np.ascontiguousarray(np.asarray(rows, dtype=np.int64))
+    out = np.empty((len(rows), W), dtype=OUT_DTYPE[pair])
+    _check(lib().oracle_sat_gen_rows(pair, mode, seed, img, value, H, W, rows.ctypes.data,
+                                     len(rows), out.ctypes.data), "oracle_sat_gen_rows")
+    return out
