@@ -1,0 +1,418 @@
+#!/usr/bin/env python3
+"""bench.py -- SAT throughput on B200 (BASELINE.json metric: Gpixels/s and
+achieved HBM GB/s vs the HBM roofline).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload NAME] [--no-sweep]
+
+Workload (N=1 headline, BASELINE.json configs[1]): the 16384 x 16384 8u->32s
+image of the size sweep, synthetic (satgen, seed 1001).  Under torchrun
+(N > 1) every rank computes its own independent 16384^2 image (image index =
+rank): the path shards by image with no data-path collective ("weak").
+
+A step = one sat_compute over the whole image (one kernel launch).  Inputs
+(268 MB in + 1.07 GB out per step) exceed the 126 MB L2, so no flush is
+needed for the headline; the sweep entries below 4096^2 flush L2 between steps.
+Timing: CUDA events on the launching stream, barrier + synchronize around the
+K timed steps, max over ranks.  rank 0 prints ONE JSON line.
+
+--impl reference times the CPU oracle (oracle/, single thread, as it stands)
+on the same workload, one full image per step (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # name: (pair, H, W, N, seed)
+    "sweep-16384sq-8u32s": (0, 16384, 16384, 1, 1001),
+    "sweep-16384sq-32f32f": (1, 16384, 16384, 1, 1001),
+    "sweep-8192sq-8u32s": (0, 8192, 8192, 1, 1001),
+    "batch-1024x1080x1920-8u32s": (0, 1080, 1920, 1024, 1002),
+    "huge-65536sq-32f32f": (1, 65536, 65536, 1, 1004),
+    "64f-16384sq": (2, 16384, 16384, 1, 1005),
+}
+DEFAULT_WORKLOAD = "sweep-16384sq-8u32s"
+PAIR_NAME = {0: "8u->32s", 1: "32f->32f", 2: "64f->64f"}
+IN_B = {0: 1, 1: 4, 2: 8}
+OUT_B = {0: 4, 1: 4, 2: 8}
+DTYPE_NAME = {0: "u32", 1: "f32", 2: "f64"}
+L2_BYTES = 126 * 1024 * 1024
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(workload):
+    """Per-launch DRAM bytes (read + write) of the SAT kernel from the committed
+    `ncu --set full` summary, if one exists for this workload."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        d = json.load(open(p))
+        e = d.get(workload)
+        return float(e["dram_bytes_per_launch"]) if e else None
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """Samples SM clock + throttle reasons via NVML during the timed region."""
+
+    def __init__(self, index: int, period_s: float = 0.002):
+        self.index, self.period = index, period_s
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.ok = False
+
+    def _run(self):
+        nv = self.nv
+        names = {
+            "hw_slowdown": getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8),
+            "hw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+            "sw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+            "sw_power_cap": getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4),
+            "hw_power_brake_slowdown": getattr(nv, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for n, bit in names.items():
+                    if r & bit:
+                        self.reasons.add(n)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples), "source": "nvml"}
+
+    def rejected(self):
+        bad = {"hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"}
+        if self.reasons & bad:
+            return True
+        if self.samples and self.max_mhz and statistics.median(self.samples) < 0.5 * self.max_mhz \
+                and not self.reasons:
+            return True
+        return False
+
+
+def host_info():
+    try:
+        model = [l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name")][0]
+    except Exception:
+        model = "?"
+    return model, os.cpu_count(), len(os.sched_getaffinity(0))
+
+
+# ---------------------------------------------------------------------------
+
+def run_reference(args, workload, rank, world):
+    """CPU oracle as the reference arm (rank 0 only)."""
+    if rank != 0:
+        return
+    import numpy as np
+
+    import oracle
+    import satgen
+
+    pair, H, W, N, seed = WORKLOADS[workload]
+    dt = {0: np.uint8, 1: np.float32, 2: np.float64}[pair]
+    img = np.empty((H, W), dtype=dt)
+    satgen.fill_host(img, seed=seed, img0=0)
+    for _ in range(args.warmup):
+        oracle.sat(img)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.sat(img)
+    el = time.perf_counter() - t0
+    px = H * W * args.steps
+    v = px / el / 1e9
+    model, ncpu, aff = host_info()
+    sample = f"one full {H}x{W} {PAIR_NAME[pair]} image per step"
+    line = {
+        "impl": "reference", "metric": "SAT Gpixels/s", "value": v, "unit": "Gpx/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": el / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "int64" if pair == 0 else ("f64" if pair == 1 else "f64x2"),
+        "data": "synthetic (satgen)",
+        "config": {"workload": workload, "pair": PAIR_NAME[pair], "H": H, "W": W, "N": 1},
+        "cpu_baseline": {"value": v, "unit": "Gpx/s", "cores": 1, "kind": "oracle",
+                         "sample": sample, "host_cpu": model, "host_cores": ncpu},
+        "e2e": {"value": v, "unit": "Gpx/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(workload, budget_s=10.0):
+    """Time the oracle (as it stands, 1 thread) on a bounded sample of the workload."""
+    import numpy as np
+
+    import oracle
+    import satgen
+
+    pair, H, W, N, seed = WORKLOADS[workload]
+    dt = {0: np.uint8, 1: np.float32, 2: np.float64}[pair]
+    # bounded sample: the first rows of the workload image, ~budget seconds of work
+    rows = min(H, 4096)
+    img = np.empty((rows, W), dtype=dt)
+    satgen.fill_host(img, seed=seed, img0=0)
+    oracle.sat(img)  # warm (page-in, lib load)
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        oracle.sat(img)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s or reps >= 64:
+            break
+    model, ncpu, aff = host_info()
+    return {"value": rows * W * reps / el / 1e9, "unit": "Gpx/s", "cores": 1, "kind": "oracle",
+            "sample": f"{reps} x the first {rows} rows ({rows}x{W}) of the workload image, "
+                      f"{el:.1f} s single-thread", "host_cpu": model, "host_cores": ncpu}
+
+
+def time_device(sat, x, out, steps, warmup, flush=None, stream=None):
+    """Per-step CUDA-event durations (ms) of sat(x -> out) on `stream`."""
+    import torch
+
+    s = stream or torch.cuda.current_stream()
+    for _ in range(warmup):
+        sat.sat(x, out=out, stream=s)
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(steps)]
+    for a, b in ev:
+        if flush is not None:
+            flush.zero_()
+        a.record(s)
+        sat.sat(x, out=out, stream=s)
+        b.record(s)
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) for a, b in ev]
+
+
+def sweep_entry(sat, satgen, torch, pair, H, W, N, seed, steps, peak):
+    dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64}[pair]
+    shape = (N, H, W) if N > 1 else (H, W)
+    x = torch.empty(shape, dtype=dt, device="cuda")
+    satgen.fill_device(x, seed=seed)
+    out = torch.empty(shape, dtype=sat.out_dtype(pair), device="cuda")
+    byts = H * W * N * (IN_B[pair] + OUT_B[pair])
+    flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device="cuda") if byts < 4 * L2_BYTES else None
+    ts = time_device(sat, x, out, steps, 3, flush)
+    ms = statistics.median(ts)
+    del x, out, flush
+    torch.cuda.empty_cache()
+    gbs = byts / (ms * 1e-3) / 1e9
+    return {"pair": PAIR_NAME[pair], "shape": f"{N}x{H}x{W}" if N > 1 else f"{H}x{W}",
+            "ms_median": round(ms, 4), "ms_min": round(min(ts), 4),
+            "gpx_s": round(H * W * N / (ms * 1e-3) / 1e9, 1), "alg_gbs": round(gbs, 1),
+            "frac_of_peak": round(gbs / peak, 3), "frac_of_8TBs": round(gbs / 8000.0, 3),
+            "l2": "flushed" if flush is not None else "inputs > L2"}
+
+
+def run_ours(args, workload, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cluster_chenwttm18_b200 as sat
+    import satgen
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    pair, H, W, N, seed = WORKLOADS[workload]
+    dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64}[pair]
+    shape = (N, H, W) if N > 1 else (H, W)
+    x = torch.empty(shape, dtype=dt, device=dev)
+    satgen.fill_device(x, seed=seed, img0=rank * N)
+    out = torch.empty(shape, dtype=sat.out_dtype(pair), device=dev)
+    plan = sat.Plan(pair, H, W, N, dev)
+    s = torch.cuda.current_stream(dev)
+    px_rank = H * W * N
+    alg_bytes = px_rank * (IN_B[pair] + OUT_B[pair])
+    peak, peak_src = peaks()
+
+    def call():
+        if N > 1:
+            es = x.element_size()
+            plan.compute_batched_ptr(x.data_ptr(), out.data_ptr(), H, W, W * es, W * 4 if pair < 2 else W * 8,
+                                     H * W * es, H * W * (OUT_B[pair]), N, s)
+        else:
+            plan.compute_ptr(x.data_ptr(), out.data_ptr(), H, W, W * IN_B[pair], W * OUT_B[pair], s)
+
+    for _ in range(args.warmup):
+        call()
+    torch.cuda.synchronize()
+
+    def timed():
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(args.steps)]
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        sampler = ClockSampler(local_rank)
+        with sampler:
+            t0.record(s)
+            for a, b in ev:
+                a.record(s)
+                call()
+                b.record(s)
+            t1.record(s)
+            torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        return t0.elapsed_time(t1), [a.elapsed_time(b) for a, b in ev], sampler
+
+    total_ms, per, sampler = timed()
+    remeasured = False
+    if sampler.rejected():
+        total_ms, per, sampler = timed()
+        remeasured = True
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms_step = total_ms / args.steps
+    value = px_rank * world * args.steps / (total_ms * 1e-3) / 1e9
+    kern_ms = statistics.mean(per)
+    achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
+
+    # end to end through the C ABI with pinned HOST buffers (H2D + SAT + D2H per step)
+    e2e = None
+    if N == 1:
+        xh = torch.empty((H, W), dtype=dt).pin_memory()
+        satgen.fill_host(xh.numpy(), seed=seed, img0=rank)
+        oh = torch.empty((H, W), dtype=sat.out_dtype(pair)).pin_memory()
+        e2e_steps = max(3, min(args.steps, 10))
+        plan.compute_host_ptr(xh.data_ptr(), oh.data_ptr(), H, W, W * IN_B[pair], W * OUT_B[pair], s)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s)
+        for _ in range(e2e_steps):
+            plan.compute_host_ptr(xh.data_ptr(), oh.data_ptr(), H, W, W * IN_B[pair], W * OUT_B[pair], s)
+        b.record(s)
+        torch.cuda.synchronize()
+        e_ms = a.elapsed_time(b)
+        if world > 1:
+            t = torch.tensor([e_ms], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms = float(t.item())
+        e2e = {"value": px_rank * world * e2e_steps / (e_ms * 1e-3) / 1e9, "unit": "Gpx/s",
+               "h2d_bytes_per_step": H * W * IN_B[pair], "d2h_bytes_per_step": H * W * OUT_B[pair],
+               "steps": e2e_steps, "path": "sat_compute_host (pinned host in/out, banded H2D/SAT/D2H overlap)"}
+        del xh, oh
+
+    if rank != 0:
+        return
+    line = {
+        "metric": "SAT Gpixels/s", "value": value, "unit": "Gpx/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": DTYPE_NAME[pair], "data": "synthetic (satgen counter-based generator)",
+        "config": {"workload": workload, "pair": PAIR_NAME[pair], "H": H, "W": W, "N": N,
+                   "images_per_rank": N, "parallelism": f"image-sharded x{world}",
+                   "l2": f"inputs larger than L2 ({alg_bytes / 1e9:.2f} GB/step vs 126 MB), no flush"},
+        "hbm_gbs": achieved, "hbm_frac_of_8TBs": achieved / 8000.0,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": ncu_traffic(workload),
+                     "kernel": "sat_tile_kernel", "peak_source": peak_src,
+                     "algorithmic_bytes_per_launch": alg_bytes,
+                     "kernel_ms_mean": kern_ms, "kernel_ms_min": min(per)},
+        "gpu_launches": args.steps,
+        "clocks": sampler.summary() | {"remeasured": remeasured},
+        "e2e": e2e,
+    }
+    if world == 1 and not args.no_sweep:
+        sweep = []
+        for (p_, h_, w_, n_) in [(0, 1024, 1024, 1), (0, 2048, 2048, 1), (0, 4096, 4096, 1),
+                                 (0, 8192, 8192, 1), (1, 1024, 1024, 1), (1, 4096, 4096, 1),
+                                 (1, 8192, 8192, 1), (1, 16384, 16384, 1), (2, 16384, 16384, 1),
+                                 (2, 4096, 65536, 1), (2, 65536, 4096, 1), (0, 4096, 65536, 1),
+                                 (1, 65536, 4096, 1), (0, 1080, 1920, 1024),
+                                 (1, 65536, 65536, 1)]:
+            try:
+                sweep.append(sweep_entry(sat, satgen, torch, p_, h_, w_, n_, 1001, 10, peak))
+            except Exception as ex:  # e.g. OOM: report, keep going
+                sweep.append({"pair": PAIR_NAME[p_], "shape": f"{n_}x{h_}x{w_}", "error": str(ex)[:200]})
+        line["sweep"] = sweep
+    if world == 1:
+        del x, out
+        torch.cuda.empty_cache()
+        line["cpu_baseline"] = cpu_baseline(workload)
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", default=DEFAULT_WORKLOAD, choices=sorted(WORKLOADS))
+    ap.add_argument("--no-sweep", action="store_true")
+    args = ap.parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, args.workload, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, args.workload, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

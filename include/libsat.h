@@ -1,0 +1,176 @@
+/* libsat.h -- C ABI of the B200-native summed-area-table library.
+ *
+ * Operation (Sec. III-A, Eq. 1; index reading R1 in DESIGN.md):
+ * the 2D inclusive summed-area table (integral image)
+ *
+ *     S(i, j) = sum_{y <= i} sum_{x <= j} A(y, x),   0 <= i < h, 0 <= j < w,
+ *
+ * of a row-major pitched image A (h rows of w elements), for the paper's type
+ * pairs T_A -> T_B (Sec. III-D):
+ *     SAT_8U_32S  : uint8  -> int32, exact, two's-complement wrap mod 2^32 (R2)
+ *     SAT_32F_32F : float  -> float  (accumulated in fp32; tolerance 1e-4 rel.)
+ *     SAT_64F_64F : double -> double (accumulated in fp64; tolerance 1e-12 rel.)
+ * Output has the same h x w shape as the input (inclusive form).
+ *
+ * Conventions (all entry points):
+ *  - Every call returns sat_status; no C++ exception crosses the ABI.  On a
+ *    non-OK status, sat_last_error() returns a thread-local detail string.
+ *  - Pointers `in`, `out`, `carry_in`, `in_band`, `out_band` are DEVICE
+ *    pointers on the plan's device (except sat_compute_host, which takes HOST
+ *    pointers).  The caller owns them; they must stay valid until the work
+ *    queued on `stream` completes.
+ *  - Pitches and strides are in BYTES, separately for input and output
+ *    (NPP nSrcStep/nDstStep style, reading R8).  Any pitch that is a multiple
+ *    of the element size and >= w * sizeof(T) is accepted; 16-byte aligned
+ *    base/pitch/stride select the TMA-fed fast path, others a generic path.
+ *  - Compute calls are asynchronous and stream-ordered: they validate
+ *    synchronously, enqueue on `stream` (a cudaStream_t passed as void*;
+ *    NULL = legacy default stream) and return without synchronising the host.
+ *    Asynchronous device faults surface at the caller's next synchronisation.
+ *  - A plan owns a workspace (look-back status words, carry payloads, a
+ *    ticket counter).  A plan must not be used by two unordered streams at
+ *    once (documented, not detected).  Workspace is never re-zeroed per call:
+ *    status words carry a per-call epoch.
+ *  - h == 0 or w == 0 (or batch == 0) is SAT_OK and a no-op.
+ *  - In-place (in == out, equal pitches/strides) is allowed for 32f/64f.
+ *    Any other overlap of input and output ranges is SAT_ERR_UNSUPPORTED.
+ *  - Validation failures return SAT_ERR_INVALID_ARGUMENT and launch nothing:
+ *    NULL pointer with non-empty extent, negative h/w/batch, pitch smaller
+ *    than w * sizeof(T) or not a multiple of sizeof(T), image stride smaller
+ *    than h * pitch or not a multiple of sizeof(T), dims above the plan
+ *    limits, `pair` different from the plan's pair.
+ */
+#ifndef LIBSAT_H
+#define LIBSAT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  SAT_OK = 0,
+  SAT_ERR_INVALID_ARGUMENT = 1,
+  SAT_ERR_UNSUPPORTED = 2,
+  SAT_ERR_CUDA = 3,
+  SAT_ERR_NCCL = 4,
+  SAT_ERR_OUT_OF_MEMORY = 5
+} sat_status;
+
+/* Type pairs T_A -> T_B. */
+typedef enum { SAT_8U_32S = 0, SAT_32F_32F = 1, SAT_64F_64F = 2 } sat_pair;
+
+typedef struct sat_plan_st* sat_plan;
+typedef struct sat_comm_st* sat_comm;
+
+/* Library version as major*10000 + minor*100 + patch. */
+int sat_version(void);
+
+/* Create a plan for `pair` on CUDA device `device`, sized for images up to
+ * max_h x max_w and batches up to max_batch (all >= 1).  Allocates the
+ * workspace on that device (see sat_plan_workspace_bytes).  *plan receives
+ * the handle; on failure *plan is NULL.
+ * Errors: INVALID_ARGUMENT (NULL plan, bad pair, non-positive limits),
+ * CUDA (no such device / not sm_100), OUT_OF_MEMORY. */
+sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t max_h, int64_t max_w,
+                           int64_t max_batch);
+
+/* Bytes of device workspace owned by the plan. */
+sat_status sat_plan_workspace_bytes(sat_plan plan, size_t* bytes);
+
+/* Free the plan and its workspace (and host-path staging buffers).  The caller
+ * must ensure no work using the plan is still pending.  NULL is a no-op. */
+sat_status sat_plan_destroy(sat_plan plan);
+
+/* SAT of one h x w image: out = S(in).  One kernel launch (single HBM pass:
+ * each input byte read once, each output byte written once). */
+sat_status sat_compute(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                       int64_t in_pitch_bytes, int64_t out_pitch_bytes, sat_pair pair, void* stream);
+
+/* SAT of `batch` independent images; image n starts at in + n*in_image_stride_bytes
+ * (resp. out + n*out_image_stride_bytes).  Carries never cross images. */
+sat_status sat_compute_batched(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                               int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                               int64_t in_image_stride_bytes, int64_t out_image_stride_bytes,
+                               int64_t batch, sat_pair pair, void* stream);
+
+/* SAT of a row band with a carry-in row: out(i, j) = carry_in[j] + S_band(i, j),
+ * where carry_in (device, w elements of T_B, contiguous) is the SAT row just
+ * above the band, S(r0 - 1, .).  carry_in == NULL means zeros (== sat_compute).
+ * This is the building block of the streamed host path and of the row-banded
+ * multi-GPU path. */
+sat_status sat_compute_band(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                            int64_t in_pitch_bytes, int64_t out_pitch_bytes, const void* carry_in,
+                            sat_pair pair, void* stream);
+
+/* End-to-end SAT of a HOST image into a HOST output (pinned memory
+ * recommended).  The image is streamed through the device in row bands:
+ * host->device copy, sat_compute_band with the previous band's last output
+ * row as carry-in, device->host copy, overlapped on internal streams.  All
+ * work is ordered after prior work on `stream`, and `stream` is made to wait
+ * for its completion; synchronise `stream` before reading `out`.
+ * Device staging buffers are allocated lazily and owned by the plan. */
+sat_status sat_compute_host(sat_plan plan, const void* in_host, void* out_host, int64_t h,
+                            int64_t w, int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                            sat_pair pair, void* stream);
+
+/* ---------------------------------------------------------------------------
+ * Multi-GPU (one process per GPU, NCCL over NVLink/NVSwitch).
+ * NCCL is loaded at run time (dlopen "libnccl.so.2"; the copy torch already
+ * loaded is reused).  Errors from NCCL map to SAT_ERR_NCCL.
+ */
+
+/* Bytes of an NCCL unique id (NCCL_UNIQUE_ID_BYTES). */
+#define SAT_COMM_ID_BYTES 128
+
+/* Rank 0 creates the id (SAT_COMM_ID_BYTES bytes at id_out) and broadcasts it
+ * out of band (e.g. torch.distributed.broadcast). */
+sat_status sat_comm_unique_id(void* id_out);
+
+/* Collective over nranks processes: create the communicator of `rank` on
+ * CUDA device `device`. */
+sat_status sat_comm_create(sat_comm* comm, const void* id, int nranks, int rank, int device);
+
+sat_status sat_comm_destroy(sat_comm comm);
+
+/* Row-banded SAT of one image of height sum_r band_h_r distributed over the
+ * communicator's ranks in rank order: rank r holds rows [r0, r0 + band_h) in
+ * in_band / out_band (device, pitched).  Each rank reduces its band's column
+ * totals, the W-vectors are all-gathered over NCCL, the exclusive prefix over
+ * lower ranks is scanned horizontally into the carry-in row S(r0 - 1, .), and
+ * the band SAT is computed with that carry-in.  All
+ * ranks must call it collectively with the same w and pair; band_h may differ
+ * per rank (0 allowed).  Ordered on `stream`. */
+sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, void* out_band,
+                            int64_t band_h, int64_t w, int64_t in_pitch_bytes,
+                            int64_t out_pitch_bytes, sat_pair pair, void* stream);
+
+/* Building blocks of sat_compute_dist (steps 1 and 3), exported so the carry
+ * algebra can be exercised without NCCL (e.g. "virtual ranks" on one GPU).
+ * Accumulator type: uint32 for SAT_8U_32S (exact mod 2^32), double
+ * (compensated sums) for the float pairs; sat_dist_acc_bytes gives its size. */
+size_t sat_dist_acc_bytes(sat_pair pair);
+
+/* acc_out[x] = sum_{y < band_h} in_band(y, x) for x < w (device, w accumulators). */
+sat_status sat_dist_colsum(sat_plan plan, const void* in_band, int64_t band_h, int64_t w,
+                           int64_t in_pitch_bytes, void* acc_out, void* stream);
+
+/* carry_out[x] = sum_{x' <= x} sum_{r < rank} gathered[r][x'] rounded once to
+ * T_B, i.e. the row S(r0 - 1, .) above rank `rank`'s band.  gathered is
+ * [nranks][w] accumulators (device), carry_out w elements of T_B (device). */
+sat_status sat_dist_carry(sat_plan plan, const void* gathered, int nranks, int rank, int64_t w,
+                          void* carry_out, void* stream);
+
+/* Static description of a status code. */
+const char* sat_status_string(sat_status s);
+
+/* Thread-local detail for the last non-OK status returned on this thread. */
+const char* sat_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LIBSAT_H */

@@ -1,0 +1,352 @@
+"""libsat: B200-native (sm_100a) summed-area tables -- Python binding.
+
+Thin ctypes marshalling over ``libsat.so`` (C ABI in ``include/libsat.h``):
+every step of the SAT runs in the library's CUDA kernels; torch is used only
+for device memory, streams and process groups.  There is no CPU fallback: if
+the extension is missing or the device is not a B200 the calls raise.
+
+    S(i, j) = sum_{y <= i} sum_{x <= j} A(y, x)        (Eq. 1)
+
+Type pairs: uint8 -> int32 (wrap mod 2^32), float32 -> float32,
+float64 -> float64.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+
+__all__ = ["SatError", "Plan", "sat", "sat_host", "SatComm", "sat_dist", "band_partition",
+           "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "lib", "LIB_PATH"]
+
+PAIR_8U_32S, PAIR_32F_32F, PAIR_64F_64F = 0, 1, 2
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsat.so")
+COMM_ID_BYTES = 128
+
+_lib = None
+_lock = threading.Lock()
+
+
+class SatError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        self.status = status
+        super().__init__(f"{where}: {_status_name(status)}: {detail}")
+
+
+def _status_name(s: int) -> str:
+    return lib().sat_status_string(s).decode()
+
+
+def lib():
+    """ctypes handle of libsat.so; raises if the extension was not built."""
+    global _lib
+    if _lib is None:
+        with _lock:
+            if _lib is None:
+                if not os.path.exists(LIB_PATH):
+                    raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build()")
+                L = ctypes.CDLL(LIB_PATH, mode=ctypes.RTLD_GLOBAL)
+                i32, i64, vp, sz = ctypes.c_int, ctypes.c_int64, ctypes.c_void_p, ctypes.c_size_t
+                sigs = {
+                    "sat_version": ([], i32),
+                    "sat_plan_create": ([ctypes.POINTER(vp), i32, i32, i64, i64, i64], i32),
+                    "sat_plan_workspace_bytes": ([vp, ctypes.POINTER(sz)], i32),
+                    "sat_plan_destroy": ([vp], i32),
+                    "sat_compute": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
+                    "sat_compute_batched": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i64, i32, vp], i32),
+                    "sat_compute_band": ([vp, vp, vp, i64, i64, i64, i64, vp, i32, vp], i32),
+                    "sat_compute_host": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
+                    "sat_comm_unique_id": ([vp], i32),
+                    "sat_comm_create": ([ctypes.POINTER(vp), vp, i32, i32, i32], i32),
+                    "sat_comm_destroy": ([vp], i32),
+                    "sat_compute_dist": ([vp, vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
+                    "sat_dist_acc_bytes": ([i32], sz),
+                    "sat_dist_colsum": ([vp, vp, i64, i64, i64, vp, vp], i32),
+                    "sat_dist_carry": ([vp, vp, i32, i32, i64, vp, vp], i32),
+                    "sat_status_string": ([i32], ctypes.c_char_p),
+                    "sat_last_error": ([], ctypes.c_char_p),
+                }
+                for name, (args, res) in sigs.items():
+                    f = getattr(L, name)
+                    f.argtypes = args
+                    f.restype = res
+                _lib = L
+    return _lib
+
+
+def _check(status: int, where: str):
+    if status != 0:
+        raise SatError(status, where, lib().sat_last_error().decode())
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def pair_of_dtype(dtype) -> int:
+    torch = _torch()
+    m = {torch.uint8: PAIR_8U_32S, torch.float32: PAIR_32F_32F, torch.float64: PAIR_64F_64F}
+    if dtype not in m:
+        raise TypeError(f"unsupported input dtype {dtype}; expected uint8, float32 or float64")
+    return m[dtype]
+
+
+def out_dtype(pair: int):
+    torch = _torch()
+    return {PAIR_8U_32S: torch.int32, PAIR_32F_32F: torch.float32, PAIR_64F_64F: torch.float64}[pair]
+
+
+def _stream_ptr(stream, device):
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream(device)
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+class Plan:
+    """A libsat plan: a pair, size limits and the look-back workspace."""
+
+    def __init__(self, pair: int, max_h: int, max_w: int, max_batch: int = 1, device=None):
+        torch = _torch()
+        dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        self.device = dev
+        self.pair, self.max_h, self.max_w, self.max_batch = pair, max_h, max_w, max_batch
+        h = ctypes.c_void_p()
+        _check(lib().sat_plan_create(ctypes.byref(h), dev.index, pair, max_h, max_w, max_batch),
+               "sat_plan_create")
+        self._h = h
+
+    @property
+    def handle(self):
+        return self._h
+
+    def workspace_bytes(self) -> int:
+        n = ctypes.c_size_t()
+        _check(lib().sat_plan_workspace_bytes(self._h, ctypes.byref(n)), "sat_plan_workspace_bytes")
+        return n.value
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            lib().sat_plan_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def fits(self, h, w, batch=1) -> bool:
+        return h <= self.max_h and w <= self.max_w and batch <= self.max_batch
+
+    # -- raw pointer calls (sizes in elements, pitches in bytes) ---------------
+    def compute_ptr(self, inp: int, out: int, h: int, w: int, in_pitch: int, out_pitch: int,
+                    stream=None):
+        _check(lib().sat_compute(self._h, inp, out, h, w, in_pitch, out_pitch, self.pair,
+                                 _stream_ptr(stream, self.device)), "sat_compute")
+
+    def compute_batched_ptr(self, inp, out, h, w, in_pitch, out_pitch, in_is, out_is, batch,
+                            stream=None):
+        _check(lib().sat_compute_batched(self._h, inp, out, h, w, in_pitch, out_pitch, in_is,
+                                         out_is, batch, self.pair, _stream_ptr(stream, self.device)),
+               "sat_compute_batched")
+
+    def compute_band_ptr(self, inp, out, h, w, in_pitch, out_pitch, carry_in, stream=None):
+        _check(lib().sat_compute_band(self._h, inp, out, h, w, in_pitch, out_pitch, carry_in,
+                                      self.pair, _stream_ptr(stream, self.device)),
+               "sat_compute_band")
+
+    def compute_host_ptr(self, inp, out, h, w, in_pitch, out_pitch, stream=None):
+        _check(lib().sat_compute_host(self._h, inp, out, h, w, in_pitch, out_pitch, self.pair,
+                                      _stream_ptr(stream, self.device)), "sat_compute_host")
+
+
+_plans: dict = {}
+
+
+def _plan_for(device, pair, h, w, batch) -> Plan:
+    key = (device.index, pair)
+    p = _plans.get(key)
+    if p is None or not p.fits(h, w, batch):
+        if p is not None:
+            _torch().cuda.synchronize(device)
+            # grow within the same order of magnitude of workspace, else size to the request
+            gh, gw, gb = max(h, p.max_h), max(w, p.max_w), max(batch, p.max_batch)
+            if gh * gw * gb <= 2 * max(h * w * batch, p.max_h * p.max_w * p.max_batch):
+                h, w, batch = gh, gw, gb
+            p.close()
+        p = Plan(pair, h, w, batch, device)
+        _plans[key] = p
+    return p
+
+
+def _row_layout(t):
+    if t.dim() not in (2, 3):
+        raise ValueError("expected a [H, W] or [N, H, W] tensor")
+    if t.stride(-1) != 1:
+        raise ValueError("the last dimension must be contiguous (stride 1)")
+    es = t.element_size()
+    H, W = t.shape[-2], t.shape[-1]
+    pitch = t.stride(-2) * es if H > 1 else max(W * es, t.stride(-2) * es)
+    img = t.stride(0) * es if t.dim() == 3 else H * pitch
+    return pitch, img
+
+
+def sat(x, out=None, plan: Plan | None = None, stream=None):
+    """Inclusive SAT of a CUDA tensor [H, W] or [N, H, W] (uint8/float32/float64).
+
+    Returns ``out`` (allocated if None: int32 / float32 / float64)."""
+    torch = _torch()
+    if not x.is_cuda:
+        raise ValueError("sat() needs a CUDA tensor (use sat_host for host arrays)")
+    pair = pair_of_dtype(x.dtype)
+    if out is None:
+        out = torch.empty(x.shape, dtype=out_dtype(pair), device=x.device)
+    elif out.dtype != out_dtype(pair) or out.shape != x.shape or out.device != x.device:
+        raise ValueError("out has the wrong dtype/shape/device")
+    H, W = x.shape[-2], x.shape[-1]
+    N = x.shape[0] if x.dim() == 3 else 1
+    if H == 0 or W == 0 or N == 0:
+        return out
+    ip, iis = _row_layout(x)
+    op, ois = _row_layout(out)
+    p = plan if plan is not None else _plan_for(x.device, pair, H, W, N)
+    if x.dim() == 3 and N > 1:
+        p.compute_batched_ptr(x.data_ptr(), out.data_ptr(), H, W, ip, op, iis, ois, N, stream)
+    else:
+        p.compute_ptr(x.data_ptr(), out.data_ptr(), H, W, ip, op, stream)
+    return out
+
+
+def sat_band(x, carry_in=None, out=None, plan: Plan | None = None, stream=None):
+    """SAT of a row band given the SAT row above it (carry_in: [W] of the output dtype)."""
+    torch = _torch()
+    pair = pair_of_dtype(x.dtype)
+    if out is None:
+        out = torch.empty(x.shape, dtype=out_dtype(pair), device=x.device)
+    H, W = x.shape
+    if H == 0 or W == 0:
+        return out
+    ip, _ = _row_layout(x)
+    op, _ = _row_layout(out)
+    cptr = None
+    if carry_in is not None:
+        if carry_in.dtype != out_dtype(pair) or carry_in.numel() < W or not carry_in.is_contiguous():
+            raise ValueError("carry_in must be a contiguous [W] tensor of the output dtype")
+        cptr = carry_in.data_ptr()
+    p = plan if plan is not None else _plan_for(x.device, pair, H, W, 1)
+    p.compute_band_ptr(x.data_ptr(), out.data_ptr(), H, W, ip, op, cptr, stream)
+    return out
+
+
+def sat_host(x, out=None, plan: Plan | None = None, device=None, stream=None):
+    """End-to-end SAT of a HOST (CPU, ideally pinned) tensor into a host tensor.
+
+    Streams row bands through the GPU (H2D, SAT with carry-in, D2H overlapped);
+    returns after synchronising the stream."""
+    torch = _torch()
+    if x.is_cuda:
+        raise ValueError("sat_host() takes a host tensor")
+    pair = pair_of_dtype(x.dtype)
+    if out is None:
+        out = torch.empty(x.shape, dtype=out_dtype(pair), pin_memory=x.is_pinned())
+    dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+    H, W = x.shape
+    if H == 0 or W == 0:
+        return out
+    ip, _ = _row_layout(x)
+    op, _ = _row_layout(out)
+    p = plan if plan is not None else _plan_for(dev, pair, H, W, 1)
+    s = stream if stream is not None else torch.cuda.current_stream(dev)
+    p.compute_host_ptr(x.data_ptr(), out.data_ptr(), H, W, ip, op, s)
+    s.synchronize()
+    return out
+
+
+# ---------------------------------------------------------------------------
+# Multi-GPU
+
+def band_partition(H: int, nranks: int, rank: int):
+    """Rows [r0, r1) of rank `rank` (reading R17: the first H mod P ranks get one extra row)."""
+    base, extra = divmod(H, nranks)
+    r0 = rank * base + min(rank, extra)
+    return r0, r0 + base + (1 if rank < extra else 0)
+
+
+class SatComm:
+    """NCCL communicator for sat_dist, bootstrapped over a torch process group."""
+
+    def __init__(self, group=None, device=None):
+        torch = _torch()
+        import torch.distributed as dist
+
+        self.rank = dist.get_rank(group)
+        self.nranks = dist.get_world_size(group)
+        dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        self.device = dev
+        buf = (ctypes.c_uint8 * COMM_ID_BYTES)()
+        if self.rank == 0:
+            _check(lib().sat_comm_unique_id(buf), "sat_comm_unique_id")
+        t = torch.tensor(list(bytes(buf)), dtype=torch.uint8)
+        if dist.get_backend(group) == "nccl":
+            t = t.to(dev)
+        dist.broadcast(t, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+        raw = bytes(t.cpu().tolist())
+        idbuf = (ctypes.c_uint8 * COMM_ID_BYTES).from_buffer_copy(raw)
+        h = ctypes.c_void_p()
+        _check(lib().sat_comm_create(ctypes.byref(h), idbuf, self.nranks, self.rank, dev.index),
+               "sat_comm_create")
+        self._h = h
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            lib().sat_comm_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def sat_dist(band, comm: SatComm, out=None, plan: Plan | None = None, stream=None):
+    """Row-banded SAT: `band` holds this rank's rows of one image (ranks in order)."""
+    torch = _torch()
+    pair = pair_of_dtype(band.dtype)
+    if out is None:
+        out = torch.empty(band.shape, dtype=out_dtype(pair), device=band.device)
+    H, W = band.shape
+    ip, _ = _row_layout(band) if H > 0 else (W * band.element_size(), 0)
+    op, _ = _row_layout(out) if H > 0 else (W * out.element_size(), 0)
+    p = plan if plan is not None else _plan_for(band.device, pair, max(H, 1), W, 1)
+    _check(lib().sat_compute_dist(p.handle, comm._h, band.data_ptr() if H else None,
+                                  out.data_ptr() if H else None, H, W, ip, op, pair,
+                                  _stream_ptr(stream, band.device)), "sat_compute_dist")
+    return out
+
+
+def dist_colsum(band, plan: Plan | None = None, stream=None):
+    """Step 1 of sat_dist: the band's column totals (uint32 or float64 [W])."""
+    torch = _torch()
+    pair = pair_of_dtype(band.dtype)
+    H, W = band.shape
+    acc = torch.empty(W, dtype=torch.int32 if pair == PAIR_8U_32S else torch.float64, device=band.device)
+    ip = band.stride(0) * band.element_size() if H > 1 else W * band.element_size()
+    p = plan if plan is not None else _plan_for(band.device, pair, max(H, 1), W, 1)
+    _check(lib().sat_dist_colsum(p.handle, band.data_ptr() if H else None, H, W, ip,
+                                 acc.data_ptr(), _stream_ptr(stream, band.device)), "sat_dist_colsum")
+    return acc
+
+
+def dist_carry(gathered, rank: int, pair: int, plan: Plan | None = None, stream=None):
+    """Step 3 of sat_dist: carry row S(r0-1, .) for `rank` from the [P, W] gathered totals."""
+    torch = _torch()
+    P, W = gathered.shape
+    carry = torch.empty(W, dtype=out_dtype(pair), device=gathered.device)
+    p = plan if plan is not None else _plan_for(gathered.device, pair, 1, W, 1)
+    _check(lib().sat_dist_carry(p.handle, gathered.contiguous().data_ptr(), P, rank, W,
+                                carry.data_ptr(), _stream_ptr(stream, gathered.device)),
+           "sat_dist_carry")
+    return carry

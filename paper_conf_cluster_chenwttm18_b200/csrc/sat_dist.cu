@@ -1,0 +1,371 @@
+// sat_dist.cu -- row-banded multi-GPU SAT (one process per GPU, NCCL).
+//
+// Rank r holds rows [r0, r1) of one image.  Its output needs the carry row
+// S(r0-1, x) = sum_{x' <= x} sum_{y < r0} A(y, x')  (Eq. 1).
+// Plan ("reduce-first"):
+//   1. sat_colsum_kernel    : raw column totals of the local band (accumulated
+//                              in u32 for 8u, compensated fp64 for 32f/64f);
+//   2. ncclAllGather         : every rank receives all ranks' W-vectors over
+//                              NVLink/NVSwitch (the one data exchange);
+//   3. sat_band_carry_kernel : exclusive prefix over lower ranks, then the
+//                              horizontal inclusive prefix over x, rounded
+//                              once to T_B -> the carry-in row;
+//   4. sat_tile_kernel       : the band's SAT with that carry-in on its top
+//                              tile row (fused carry-add: no extra pass).
+// The paper itself is single-node; this path is the build's
+// horizontal-scaling extension.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <mutex>
+
+#include "nccl.h"
+#include "sat_internal.h"
+
+namespace sat {
+
+// ---------------------------------------------------------------------------
+// NCCL, loaded at run time (reuses the libnccl.so.2 torch already loaded).
+struct NcclApi {
+  bool ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+static NcclApi& nccl() {
+  static NcclApi api;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    const char* env = getenv("SAT_NCCL_LIBRARY");
+    void* h = env ? dlopen(env, RTLD_NOW | RTLD_GLOBAL) : nullptr;
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return;
+    api.GetUniqueId = (decltype(api.GetUniqueId))dlsym(h, "ncclGetUniqueId");
+    api.CommInitRank = (decltype(api.CommInitRank))dlsym(h, "ncclCommInitRank");
+    api.CommDestroy = (decltype(api.CommDestroy))dlsym(h, "ncclCommDestroy");
+    api.AllGather = (decltype(api.AllGather))dlsym(h, "ncclAllGather");
+    api.GetErrorString = (decltype(api.GetErrorString))dlsym(h, "ncclGetErrorString");
+    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.AllGather &&
+             api.GetErrorString;
+  });
+  return api;
+}
+
+static sat_status nccl_fail(ncclResult_t r, const char* what) {
+  return fail(SAT_ERR_NCCL, "%s: %s", what, nccl().GetErrorString ? nccl().GetErrorString(r) : "?");
+}
+
+// ---------------------------------------------------------------------------
+// Kernels
+
+constexpr int kColsumThreads = 256;
+
+template <typename TA, typename ACC>
+__global__ void sat_colsum_kernel(const char* __restrict__ in, int64_t h, int64_t w, int64_t pitch,
+                                  int64_t rows_per_split, ACC* __restrict__ partial) {
+  const int64_t x = (int64_t)blockIdx.x * kColsumThreads + threadIdx.x;
+  const int64_t y0 = (int64_t)blockIdx.y * rows_per_split;
+  const int64_t y1 = min(h, y0 + rows_per_split);
+  if (x >= w) return;
+  ACC s = ACC(0), comp = ACC(0);
+  for (int64_t y = y0; y < y1; ++y) {
+    const ACC v = (ACC)reinterpret_cast<const TA*>(in + y * pitch)[x];
+    if constexpr (sizeof(ACC) == 8) {  // Kahan-Babuska (Neumaier) compensated sum
+      const ACC t = s + v;
+      comp += (fabs(s) >= fabs(v)) ? ((s - t) + v) : ((v - t) + s);
+      s = t;
+    } else {
+      s += v;  // u32, exact mod 2^32
+    }
+  }
+  partial[(int64_t)blockIdx.y * w + x] = s + comp;
+}
+
+template <typename ACC>
+__global__ void sat_colsum_reduce_kernel(const ACC* __restrict__ partial, int splits, int64_t w,
+                                         ACC* __restrict__ out) {
+  const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (x >= w) return;
+  ACC s = ACC(0), comp = ACC(0);
+  for (int k = 0; k < splits; ++k) {
+    const ACC v = partial[(int64_t)k * w + x];
+    if constexpr (sizeof(ACC) == 8) {
+      const ACC t = s + v;
+      comp += (fabs(s) >= fabs(v)) ? ((s - t) + v) : ((v - t) + s);
+      s = t;
+    } else {
+      s += v;
+    }
+  }
+  out[x] = s + comp;
+}
+
+// One CTA: c(x) = sum_{r' < rank} gathered[r'][x]; carry(x) = sum_{x' <= x} c(x').
+constexpr int kCarryThreads = 1024;
+
+template <typename ACC, typename TB>
+__global__ void __launch_bounds__(kCarryThreads)
+    sat_band_carry_kernel(const ACC* __restrict__ gathered, int rank, int64_t w, TB* __restrict__ carry) {
+  __shared__ ACC part[kCarryThreads];
+  const int64_t seg = (w + kCarryThreads - 1) / kCarryThreads;
+  const int64_t x0 = (int64_t)threadIdx.x * seg;
+  const int64_t x1 = min(w, x0 + seg);
+  // pass 1: segment total of c(x)
+  ACC tot = ACC(0), totc = ACC(0);
+  for (int64_t x = x0; x < x1; ++x) {
+    ACC c = ACC(0);
+    for (int r = 0; r < rank; ++r) c += gathered[(int64_t)r * w + x];
+    if constexpr (sizeof(ACC) == 8) {
+      const ACC t = tot + c;
+      totc += (fabs(tot) >= fabs(c)) ? ((tot - t) + c) : ((c - t) + tot);
+      tot = t;
+    } else {
+      tot += c;
+    }
+  }
+  part[threadIdx.x] = tot + totc;
+  __syncthreads();
+  // exclusive scan of segment totals (serial by thread 0: 1024 adds)
+  if (threadIdx.x == 0) {
+    ACC run = ACC(0), runc = ACC(0);
+    for (int i = 0; i < kCarryThreads; ++i) {
+      const ACC v = part[i];
+      part[i] = run + runc;
+      if constexpr (sizeof(ACC) == 8) {
+        const ACC t = run + v;
+        runc += (fabs(run) >= fabs(v)) ? ((run - t) + v) : ((v - t) + run);
+        run = t;
+      } else {
+        run += v;
+      }
+    }
+  }
+  __syncthreads();
+  // pass 2: inclusive prefix within the segment, rounded once to T_B
+  ACC run = part[threadIdx.x], runc = ACC(0);
+  for (int64_t x = x0; x < x1; ++x) {
+    ACC c = ACC(0);
+    for (int r = 0; r < rank; ++r) c += gathered[(int64_t)r * w + x];
+    if constexpr (sizeof(ACC) == 8) {
+      const ACC t = run + c;
+      runc += (fabs(run) >= fabs(c)) ? ((run - t) + c) : ((c - t) + run);
+      run = t;
+    } else {
+      run += c;
+    }
+    carry[x] = (TB)(run + runc);
+  }
+}
+
+size_t acc_size(sat_pair p) { return p == SAT_8U_32S ? 4 : 8; }
+
+// ---------------------------------------------------------------------------
+
+struct DistBufs {
+  int64_t w = 0;
+  int nranks = 0;
+  int splits = 0;
+  void* partial = nullptr;   // [splits][w] ACC
+  void* local = nullptr;     // [w] ACC
+  void* gathered = nullptr;  // [nranks][w] ACC
+  void* carry = nullptr;     // [w] TB
+};
+
+sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t pitch,
+                  void* partial, int splits, void* out, cudaStream_t s) {
+  if (h <= 0) {
+    cudaError_t e = cudaMemsetAsync(out, 0, (size_t)w * acc_size(pair), s);
+    return e == cudaSuccess ? SAT_OK : cuda_fail(e, "cudaMemsetAsync(colsum)");
+  }
+  const int64_t rps = (h + splits - 1) / splits;
+  const int used = (int)((h + rps - 1) / rps);
+  dim3 grid((unsigned)((w + kColsumThreads - 1) / kColsumThreads), (unsigned)used);
+  const char* p = static_cast<const char*>(in);
+  switch (pair) {
+    case SAT_8U_32S:
+      sat_colsum_kernel<uint8_t, uint32_t><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (uint32_t*)partial);
+      sat_colsum_reduce_kernel<uint32_t><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((uint32_t*)partial, used, w, (uint32_t*)out);
+      break;
+    case SAT_32F_32F:
+      sat_colsum_kernel<float, double><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
+      sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
+      break;
+    case SAT_64F_64F:
+      sat_colsum_kernel<double, double><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
+      sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
+      break;
+  }
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "sat_colsum_kernel launch");
+}
+
+sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, void* carry,
+                      cudaStream_t s) {
+  switch (pair) {
+    case SAT_8U_32S:
+      sat_band_carry_kernel<uint32_t, uint32_t><<<1, kCarryThreads, 0, s>>>((const uint32_t*)gathered, rank, w, (uint32_t*)carry);
+      break;
+    case SAT_32F_32F:
+      sat_band_carry_kernel<double, float><<<1, kCarryThreads, 0, s>>>((const double*)gathered, rank, w, (float*)carry);
+      break;
+    case SAT_64F_64F:
+      sat_band_carry_kernel<double, double><<<1, kCarryThreads, 0, s>>>((const double*)gathered, rank, w, (double*)carry);
+      break;
+  }
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "sat_band_carry_kernel launch");
+}
+
+}  // namespace sat
+
+using namespace sat;
+
+struct sat_comm_st {
+  ncclComm_t comm = nullptr;
+  int nranks = 0, rank = 0, device = 0;
+  DistBufs bufs;
+};
+
+static void free_bufs(DistBufs& b) {
+  if (b.partial) cudaFree(b.partial);
+  if (b.local) cudaFree(b.local);
+  if (b.gathered) cudaFree(b.gathered);
+  if (b.carry) cudaFree(b.carry);
+  b = DistBufs();
+}
+
+static sat_status ensure_bufs(DistBufs& b, int64_t w, int nranks) {
+  if (b.w >= w && b.nranks >= nranks) return SAT_OK;
+  free_bufs(b);
+  b.w = w;
+  b.nranks = nranks;
+  b.splits = 64;
+  cudaError_t e = cudaMalloc(&b.partial, (size_t)b.splits * w * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&b.local, (size_t)w * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&b.gathered, (size_t)nranks * w * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&b.carry, (size_t)w * 8);
+  if (e != cudaSuccess) {
+    free_bufs(b);
+    return cuda_fail(e, "dist buffers");
+  }
+  return SAT_OK;
+}
+
+extern "C" {
+
+sat_status sat_comm_unique_id(void* id_out) {
+  if (!id_out) return fail(SAT_ERR_INVALID_ARGUMENT, "id_out is NULL");
+  if (!nccl().ok) return fail(SAT_ERR_NCCL, "libnccl.so.2 could not be loaded");
+  ncclUniqueId id;
+  ncclResult_t r = nccl().GetUniqueId(&id);
+  if (r != ncclSuccess) return nccl_fail(r, "ncclGetUniqueId");
+  static_assert(sizeof(id) == SAT_COMM_ID_BYTES, "unique id size");
+  memcpy(id_out, &id, sizeof(id));
+  return SAT_OK;
+}
+
+sat_status sat_comm_create(sat_comm* comm, const void* id, int nranks, int rank, int device) {
+  if (!comm || !id) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
+  *comm = nullptr;
+  if (nranks < 1 || rank < 0 || rank >= nranks)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "bad rank %d of %d", rank, nranks);
+  if (!nccl().ok) return fail(SAT_ERR_NCCL, "libnccl.so.2 could not be loaded");
+  DeviceGuard g(device);
+  ncclUniqueId uid;
+  memcpy(&uid, id, sizeof(uid));
+  sat_comm_st* c = new sat_comm_st();
+  c->nranks = nranks;
+  c->rank = rank;
+  c->device = device;
+  ncclResult_t r = nccl().CommInitRank(&c->comm, nranks, uid, rank);
+  if (r != ncclSuccess) {
+    delete c;
+    return nccl_fail(r, "ncclCommInitRank");
+  }
+  *comm = c;
+  return SAT_OK;
+}
+
+sat_status sat_comm_destroy(sat_comm comm) {
+  if (!comm) return SAT_OK;
+  DeviceGuard g(comm->device);
+  cudaDeviceSynchronize();
+  free_bufs(comm->bufs);
+  if (comm->comm) nccl().CommDestroy(comm->comm);
+  delete comm;
+  return SAT_OK;
+}
+
+// Building blocks of sat_compute_dist, exported so that the carry algebra can
+// be exercised on one GPU with "virtual ranks" (tests/test_dist_gpu.py).
+size_t sat_dist_acc_bytes(sat_pair pair) { return acc_size(pair); }
+
+sat_status sat_dist_colsum(sat_plan plan, const void* in_band, int64_t band_h, int64_t w,
+                           int64_t in_pitch_bytes, void* acc_out, void* stream) {
+  if (!plan || !acc_out || (band_h > 0 && !in_band))
+    return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (band_h < 0 || w <= 0 || w > plan->max_w)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "bad extent");
+  if (in_pitch_bytes < w * (int64_t)in_size(plan->pair))
+    return fail(SAT_ERR_INVALID_ARGUMENT, "bad pitch");
+  DeviceGuard g(plan->device);
+  void* partial = nullptr;
+  cudaError_t e = cudaMallocAsync(&partial, (size_t)64 * w * 8, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMallocAsync");
+  sat_status st = colsum(plan->pair, in_band, band_h, w, in_pitch_bytes, partial, 64, acc_out,
+                         (cudaStream_t)stream);
+  cudaFreeAsync(partial, (cudaStream_t)stream);
+  return st;
+}
+
+sat_status sat_dist_carry(sat_plan plan, const void* gathered, int nranks, int rank, int64_t w,
+                          void* carry_out, void* stream) {
+  if (!plan || !gathered || !carry_out) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (nranks < 1 || rank < 0 || rank >= nranks || w <= 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "bad rank/extent");
+  DeviceGuard g(plan->device);
+  return band_carry(plan->pair, gathered, rank, w, carry_out, (cudaStream_t)stream);
+}
+
+sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, void* out_band,
+                            int64_t band_h, int64_t w, int64_t in_pitch_bytes,
+                            int64_t out_pitch_bytes, sat_pair pair, void* stream) {
+  if (!comm) return fail(SAT_ERR_INVALID_ARGUMENT, "comm is NULL");
+  if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (w <= 0) return fail(SAT_ERR_INVALID_ARGUMENT, "w must be positive for a collective call");
+  bool empty = false;
+  if (band_h > 0) {
+    sat_status st = validate(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
+                             band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1, pair, &empty);
+    if (st != SAT_OK) return st;
+  } else if (band_h < 0) {
+    return fail(SAT_ERR_INVALID_ARGUMENT, "negative band height");
+  } else if (pair != plan->pair || w > plan->max_w) {
+    return fail(SAT_ERR_INVALID_ARGUMENT, "pair/extent does not match the plan");
+  }
+  DeviceGuard g(plan->device);
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  DistBufs& b = comm->bufs;
+  sat_status st = ensure_bufs(b, w, comm->nranks);
+  if (st != SAT_OK) return st;
+  st = colsum(pair, in_band, band_h, w, in_pitch_bytes, b.partial, b.splits, b.local, s);
+  if (st != SAT_OK) return st;
+  const ncclDataType_t dt = pair == SAT_8U_32S ? ncclUint32 : ncclFloat64;
+  ncclResult_t r = nccl().AllGather(b.local, b.gathered, (size_t)w, dt, comm->comm, s);
+  if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
+  st = band_carry(pair, b.gathered, comm->rank, w, b.carry, s);
+  if (st != SAT_OK) return st;
+  if (band_h == 0) return SAT_OK;
+  return launch(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
+                band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1,
+                comm->rank > 0 ? b.carry : nullptr, s);
+}
+
+}  // extern "C"

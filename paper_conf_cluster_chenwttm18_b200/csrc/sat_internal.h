@@ -1,0 +1,63 @@
+// sat_internal.h -- private declarations shared by the libsat host runtime
+// translation units (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/libsat.h"
+
+namespace sat {
+struct HostPath;
+}
+
+struct sat_plan_st {
+  int device = 0;
+  sat_pair pair = SAT_8U_32S;
+  int64_t max_h = 0, max_w = 0, max_batch = 0;
+  int num_sms = 0;
+  int ctas_per_sm[3][4] = {};  // [pair][mode: bit0 TMA, bit1 vector out]
+  int64_t max_tiles = 0;       // capacity of the look-back workspace in tiles
+  void* ws = nullptr;
+  size_t ws_bytes = 0;
+  unsigned long long* counter = nullptr;  // ticket counter
+  uint32_t* flags = nullptr;              // status words
+  void* payload = nullptr;                // aggregate / inclusive carries
+  uint32_t epoch = 0;
+  uint64_t ticket_base = 0;
+  uint64_t launches = 0;
+  // streamed host path (lazily allocated)
+  sat::HostPath* host = nullptr;
+};
+
+namespace sat {
+
+sat_status fail(sat_status s, const char* fmt, ...);
+sat_status cuda_fail(cudaError_t e, const char* what);
+int getenv_int(const char* name, int dflt);
+size_t in_size(sat_pair p);
+size_t out_size(sat_pair p);
+int tile_w(sat_pair p);
+int tile_h(sat_pair p);
+
+sat_status validate(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
+                    int64_t op, int64_t iis, int64_t ois, int64_t batch, sat_pair pair,
+                    bool* empty);
+sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
+                  int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
+                  cudaStream_t stream);
+void host_path_release(sat_plan_st* pl);
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+    else prev = -1;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace sat

@@ -1,0 +1,405 @@
+// sat_runtime.cu -- libsat host runtime: plans, validation, tensor-map
+// encoding, epoch/ticket workspace management, launches, the streamed host
+// path.  C ABI declared in include/libsat.h.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <mutex>
+
+#include "../../include/libsat.h"
+#include "sat_internal.h"
+#include "sat_kernel.cuh"
+
+namespace {
+
+thread_local char g_last_error[512] = "";
+
+}  // namespace
+
+namespace sat {
+
+sat_status fail(sat_status s, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_last_error, sizeof(g_last_error), fmt, ap);
+  va_end(ap);
+  return s;
+}
+
+sat_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(e == cudaErrorMemoryAllocation ? SAT_ERR_OUT_OF_MEMORY : SAT_ERR_CUDA, "%s: %s (%s)",
+              what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+size_t in_size(sat_pair p) { return p == SAT_8U_32S ? 1 : (p == SAT_32F_32F ? 4 : 8); }
+size_t out_size(sat_pair p) { return p == SAT_64F_64F ? 8 : 4; }
+int tile_w(sat_pair p) {
+  return p == SAT_8U_32S ? Cfg<P8U32S>::TW : (p == SAT_32F_32F ? Cfg<P32F32F>::TW : Cfg<P64F64F>::TW);
+}
+int tile_h(sat_pair p) {
+  return p == SAT_8U_32S ? Cfg<P8U32S>::TH : (p == SAT_32F_32F ? Cfg<P32F32F>::TH : Cfg<P64F64F>::TH);
+}
+
+// ---------------------------------------------------------------------------
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda).
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn get_encode() {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  });
+  return fn;
+}
+
+template <int P>
+static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
+                           int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
+                           const void* carry_in, cudaStream_t stream) {
+  using C = Cfg<P>;
+  const bool tma = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
+                   getenv_int("SAT_FORCE_GENERIC", 0) == 0;
+  const bool vec = ((uintptr_t)out % 16 == 0) && (op % 16 == 0) && (batch == 1 || ois % 16 == 0);
+  KParams kp;
+  kp.in = static_cast<const char*>(in);
+  kp.out = static_cast<char*>(out);
+  kp.H = h;
+  kp.W = w;
+  kp.in_pitch = ip;
+  kp.out_pitch = op;
+  kp.in_img_stride = iis;
+  kp.out_img_stride = ois;
+  kp.bands_per_image = (h + C::TH - 1) / C::TH;
+  kp.total_bands = kp.bands_per_image * batch;
+  kp.nchunks = (int32_t)((w + C::TW - 1) / C::TW);
+  kp.carry_in = carry_in;
+  if (kp.total_bands * kp.nchunks > pl->max_tiles)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "problem needs %lld tiles, plan holds %lld",
+                (long long)(kp.total_bands * kp.nchunks), (long long)pl->max_tiles);
+
+  CUtensorMap map;
+  memset(&map, 0, sizeof(map));
+  if (tma) {
+    EncodeTiledFn enc = get_encode();
+    if (!enc) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    const CUtensorMapDataType dt = P == P8U32S    ? CU_TENSOR_MAP_DATA_TYPE_UINT8
+                                   : P == P32F32F ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                                  : CU_TENSOR_MAP_DATA_TYPE_FLOAT64;
+    cuuint64_t dims[3] = {(cuuint64_t)w, (cuuint64_t)h, (cuuint64_t)batch};
+    cuuint64_t strides[2] = {(cuuint64_t)ip, (cuuint64_t)(batch > 1 ? iis : ip * h)};
+    cuuint32_t box[3] = {(cuuint32_t)C::TW, (cuuint32_t)C::TH, 1};
+    cuuint32_t estr[3] = {1, 1, 1};
+    CUresult r = enc(&map, dt, 3, const_cast<void*>(in), dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  }
+
+  // Epoch: status words from earlier launches carry older epochs.
+  if (pl->epoch + 1 >= (1u << 30)) {
+    cudaError_t e = cudaMemsetAsync(pl->flags, 0, pl->max_tiles * sizeof(uint32_t), stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(flags)");
+    pl->epoch = 0;
+  }
+  kp.epoch = ++pl->epoch;
+  kp.counter = pl->counter;
+  kp.flags = pl->flags;
+  kp.payload = pl->payload;
+  kp.ticket_base = pl->ticket_base;
+
+  const int mode = (tma ? 1 : 0) | (vec ? 2 : 0);
+  const int per_sm = pl->ctas_per_sm[P][mode];
+  int64_t grid = (int64_t)pl->num_sms * std::max(per_sm, 1);
+  const int cap = getenv_int("SAT_CTAS_PER_SM", 0);
+  if (cap > 0) grid = (int64_t)pl->num_sms * std::min(cap, std::max(per_sm, 1));
+  grid = std::min<int64_t>(grid, kp.total_bands);
+  const size_t smem = sizeof(Smem<P>);
+
+  cudaError_t e;
+  switch (mode) {
+    case 0:
+      sat_tile_kernel<P, false, false><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
+      break;
+    case 1:
+      sat_tile_kernel<P, true, false><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
+      break;
+    case 2:
+      sat_tile_kernel<P, false, true><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
+      break;
+    default:
+      sat_tile_kernel<P, true, true><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
+      break;
+  }
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
+  // Every CTA draws exactly one failing ticket.
+  pl->ticket_base += (uint64_t)kp.total_bands + (uint64_t)grid;
+  pl->launches++;
+  if (getenv_int("SAT_LOG", 0))
+    fprintf(stderr, "[libsat] pair=%d %lldx%lld batch=%lld tma=%d vec=%d grid=%lld smem=%zu epoch=%u\n",
+            P, (long long)h, (long long)w, (long long)batch, (int)tma, (int)vec, (long long)grid,
+            smem, kp.epoch);
+  return SAT_OK;
+}
+
+sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
+                  int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
+                  cudaStream_t stream) {
+  switch (pl->pair) {
+    case SAT_8U_32S:
+      return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream);
+    case SAT_32F_32F:
+      return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream);
+    case SAT_64F_64F:
+      return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream);
+  }
+  return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
+}
+
+int getenv_int(const char* name, int dflt) {
+  const char* v = getenv(name);
+  return v && *v ? atoi(v) : dflt;
+}
+
+template <int P>
+static sat_status configure_t(sat_plan_st* pl) {
+  const size_t smem = sizeof(Smem<P>);
+  void (*fns[4])(CUtensorMap, KParams) = {
+      sat_tile_kernel<P, false, false>, sat_tile_kernel<P, true, false>,
+      sat_tile_kernel<P, false, true>, sat_tile_kernel<P, true, true>};
+  for (int m = 0; m < 4; ++m) {
+    cudaError_t e = cudaFuncSetAttribute(fns[m], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
+    int n = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fns[m], kThreads, smem);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
+    pl->ctas_per_sm[P][m] = n;
+  }
+  return SAT_OK;
+}
+
+sat_status configure(sat_plan_st* pl) {
+  switch (pl->pair) {
+    case SAT_8U_32S:
+      return configure_t<P8U32S>(pl);
+    case SAT_32F_32F:
+      return configure_t<P32F32F>(pl);
+    case SAT_64F_64F:
+      return configure_t<P64F64F>(pl);
+  }
+  return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
+}
+
+// ---------------------------------------------------------------------------
+// Validation (synchronous; nothing is launched on failure)
+
+static bool ranges_overlap(const void* a, size_t an, const void* b, size_t bn) {
+  const uintptr_t a0 = (uintptr_t)a, a1 = a0 + an, b0 = (uintptr_t)b, b1 = b0 + bn;
+  return a0 < b1 && b0 < a1;
+}
+
+sat_status validate(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
+                    int64_t op, int64_t iis, int64_t ois, int64_t batch, sat_pair pair,
+                    bool* empty) {
+  *empty = false;
+  if (!pl) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (pair != pl->pair)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "pair %d does not match the plan's pair %d", (int)pair,
+                (int)pl->pair);
+  if (h < 0 || w < 0 || batch < 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "negative extent (h=%lld w=%lld batch=%lld)",
+                (long long)h, (long long)w, (long long)batch);
+  if (h == 0 || w == 0 || batch == 0) {
+    *empty = true;
+    return SAT_OK;
+  }
+  if (!in || !out) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL input or output pointer");
+  if (h > pl->max_h || w > pl->max_w || batch > pl->max_batch)
+    return fail(SAT_ERR_INVALID_ARGUMENT,
+                "extent %lldx%lld batch %lld exceeds plan limits %lldx%lld batch %lld",
+                (long long)h, (long long)w, (long long)batch, (long long)pl->max_h,
+                (long long)pl->max_w, (long long)pl->max_batch);
+  const int64_t sa = (int64_t)in_size(pair), sb = (int64_t)out_size(pair);
+  if (ip < w * sa || ip % sa != 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "input pitch %lld invalid for w=%lld (elem %lld B)",
+                (long long)ip, (long long)w, (long long)sa);
+  if (op < w * sb || op % sb != 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "output pitch %lld invalid for w=%lld (elem %lld B)",
+                (long long)op, (long long)w, (long long)sb);
+  if ((uintptr_t)in % sa != 0 || (uintptr_t)out % sb != 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "pointer not aligned to its element size");
+  if (batch > 1) {
+    if (iis < h * ip || iis % sa != 0)
+      return fail(SAT_ERR_INVALID_ARGUMENT, "input image stride %lld invalid", (long long)iis);
+    if (ois < h * op || ois % sb != 0)
+      return fail(SAT_ERR_INVALID_ARGUMENT, "output image stride %lld invalid", (long long)ois);
+  }
+  // Overlap: only exact in-place for equal element sizes and layouts.
+  const size_t in_bytes = (size_t)((batch - 1) * (batch > 1 ? iis : 0) + (h - 1) * ip + w * sa);
+  const size_t out_bytes = (size_t)((batch - 1) * (batch > 1 ? ois : 0) + (h - 1) * op + w * sb);
+  if (ranges_overlap(in, in_bytes, out, out_bytes)) {
+    const bool inplace = in == out && sa == sb && ip == op && (batch == 1 || iis == ois);
+    if (!inplace)
+      return fail(SAT_ERR_UNSUPPORTED, "input and output overlap (only exact in-place for 32f/64f)");
+  }
+  return SAT_OK;
+}
+
+}  // namespace sat
+
+using namespace sat;
+
+// ===========================================================================
+// C ABI
+
+extern "C" {
+
+int sat_version(void) { return 100; }
+
+const char* sat_status_string(sat_status s) {
+  switch (s) {
+    case SAT_OK:
+      return "SAT_OK";
+    case SAT_ERR_INVALID_ARGUMENT:
+      return "SAT_ERR_INVALID_ARGUMENT";
+    case SAT_ERR_UNSUPPORTED:
+      return "SAT_ERR_UNSUPPORTED";
+    case SAT_ERR_CUDA:
+      return "SAT_ERR_CUDA";
+    case SAT_ERR_NCCL:
+      return "SAT_ERR_NCCL";
+    case SAT_ERR_OUT_OF_MEMORY:
+      return "SAT_ERR_OUT_OF_MEMORY";
+  }
+  return "SAT_ERR_UNKNOWN";
+}
+
+const char* sat_last_error(void) { return g_last_error; }
+
+sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t max_h, int64_t max_w,
+                           int64_t max_batch) {
+  if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan out-pointer is NULL");
+  *plan = nullptr;
+  if (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "unknown pair %d", (int)pair);
+  if (max_h <= 0 || max_w <= 0 || max_batch <= 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "plan limits must be positive");
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
+  if (device < 0 || device >= ndev) return fail(SAT_ERR_CUDA, "no CUDA device %d", device);
+  cudaDeviceProp prop;
+  e = cudaGetDeviceProperties(&prop, device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceProperties");
+  if (prop.major != 10 || prop.minor != 0)
+    return fail(SAT_ERR_CUDA, "device %d is sm_%d%d; libsat is built for sm_100a only", device,
+                prop.major, prop.minor);
+  int prev = 0;
+  cudaGetDevice(&prev);
+  e = cudaSetDevice(device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+
+  sat_plan_st* pl = new sat_plan_st();
+  pl->device = device;
+  pl->pair = pair;
+  pl->max_h = max_h;
+  pl->max_w = max_w;
+  pl->max_batch = max_batch;
+  pl->num_sms = prop.multiProcessorCount;
+  const int64_t TH = tile_h(pair), TW = tile_w(pair);
+  pl->max_tiles = max_batch * ((max_h + TH - 1) / TH) * ((max_w + TW - 1) / TW);
+  const size_t flags_bytes = ((size_t)pl->max_tiles * 4 + 255) / 256 * 256;
+  const size_t payload_bytes = (size_t)pl->max_tiles * 2 * TW * out_size(pair);
+  pl->ws_bytes = 256 + flags_bytes + payload_bytes;
+  sat_status st = configure(pl);
+  if (st == SAT_OK) {
+    e = cudaMalloc(&pl->ws, pl->ws_bytes);
+    if (e != cudaSuccess) st = cuda_fail(e, "cudaMalloc(workspace)");
+  }
+  if (st == SAT_OK) {
+    e = cudaMemset(pl->ws, 0, 256 + flags_bytes);
+    if (e != cudaSuccess) st = cuda_fail(e, "cudaMemset(workspace)");
+  }
+  if (st != SAT_OK) {
+    if (pl->ws) cudaFree(pl->ws);
+    delete pl;
+    cudaSetDevice(prev);
+    return st;
+  }
+  pl->counter = reinterpret_cast<unsigned long long*>(pl->ws);
+  pl->flags = reinterpret_cast<uint32_t*>(static_cast<char*>(pl->ws) + 256);
+  pl->payload = static_cast<char*>(pl->ws) + 256 + flags_bytes;
+  cudaSetDevice(prev);
+  *plan = pl;
+  return SAT_OK;
+}
+
+sat_status sat_plan_workspace_bytes(sat_plan plan, size_t* bytes) {
+  if (!plan || !bytes) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
+  *bytes = plan->ws_bytes;
+  return SAT_OK;
+}
+
+sat_status sat_plan_destroy(sat_plan plan) {
+  if (!plan) return SAT_OK;
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(plan->device);
+  host_path_release(plan);
+  if (plan->ws) cudaFree(plan->ws);
+  cudaSetDevice(prev);
+  delete plan;
+  return SAT_OK;
+}
+
+sat_status sat_compute_batched(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                               int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                               int64_t in_image_stride_bytes, int64_t out_image_stride_bytes,
+                               int64_t batch, sat_pair pair, void* stream) {
+  bool empty = false;
+  sat_status st = validate(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
+                           in_image_stride_bytes, out_image_stride_bytes, batch, pair, &empty);
+  if (st != SAT_OK || empty) return st;
+  DeviceGuard g(plan->device);
+  return launch(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
+                batch > 1 ? in_image_stride_bytes : h * in_pitch_bytes,
+                batch > 1 ? out_image_stride_bytes : h * out_pitch_bytes, batch, nullptr,
+                static_cast<cudaStream_t>(stream));
+}
+
+sat_status sat_compute(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                       int64_t in_pitch_bytes, int64_t out_pitch_bytes, sat_pair pair,
+                       void* stream) {
+  return sat_compute_batched(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
+                             h * in_pitch_bytes, h * out_pitch_bytes, 1, pair, stream);
+}
+
+sat_status sat_compute_band(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                            int64_t in_pitch_bytes, int64_t out_pitch_bytes, const void* carry_in,
+                            sat_pair pair, void* stream) {
+  bool empty = false;
+  sat_status st = validate(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
+                           h * in_pitch_bytes, h * out_pitch_bytes, 1, pair, &empty);
+  if (st != SAT_OK || empty) return st;
+  if (carry_in && (uintptr_t)carry_in % out_size(pair) != 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "carry_in not aligned to its element size");
+  DeviceGuard g(plan->device);
+  return launch(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes, h * in_pitch_bytes,
+                h * out_pitch_bytes, 1, carry_in, static_cast<cudaStream_t>(stream));
+}
+
+}  // extern "C"
