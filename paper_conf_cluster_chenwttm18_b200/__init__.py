@@ -21,7 +21,7 @@ __all__ = ["SatError", "Plan", "sat", "sat_host", "SatComm", "sat_dist", "band_p
 
 PAIR_8U_32S, PAIR_32F_32F, PAIR_64F_64F = 0, 1, 2
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsat.so")
+LIB_PATH = os.environ.get("SAT_LIBRARY") or os.path.join(_HERE, "libsat.so")
 COMM_ID_BYTES = 128
 
 _lib = None

@@ -23,19 +23,24 @@
 //       totals (Alg. 3, condition read as lane >= d, reading R10);
 //   a5  each compute warp owns RW consecutive rows and keeps a per-thread
 //       running column sum (serial scan down the rows, Alg. 2);
-//   a4  the 8 compute warps' column totals are combined in shared memory by
-//       the look-back warp (block partial-sum scan, Fig. 3c).
+//   a4  the compute warps' column totals are combined in shared memory by
+//       the look-back warps (block partial-sum scan, Fig. 3c).
 //
-// Warp roles (one CTA = 8 compute warps + 1 producer warp + 1 look-back warp):
-//   producer : draws band tickets (atomic counter => forward progress) and
-//              streams the band's tiles into an NSTAGE-deep shared-memory ring
-//              with TMA (cp.async.bulk.tensor.3d, mbarrier complete_tx), or
-//              with plain loads on the generic (unaligned) path;
-//   compute  : local pass of chunk c, then the fix-up + store of chunk c-1
-//              (so the look-back of chunk c-1 overlaps the local pass of c);
-//   look-back: per chunk, publishes the aggregate, looks back up the tile
-//              column (32 predecessors per probe), publishes the inclusive
-//              prefix and writes per-warp fix-up offsets.
+// Warp roles (one CTA = 8 compute warps + 1 producer warp + kNLB look-back
+// warps):
+//   producer : draws band tickets (atomic counter => forward progress), late
+//              enough that a drawn band is active, and streams the band's
+//              tiles into an NSTAGE-deep shared-memory ring with TMA
+//              (cp.async.bulk.tensor.3d + mbarrier complete_tx), or with plain
+//              loads on the generic (unaligned) path;
+//   compute  : pass A of chunk q (row + column scans -> the warp's column
+//              totals, row carries advanced), and, LOOK chunks later, pass B
+//              of chunk q: the same scans re-run from the still-resident smem
+//              tile plus the fix-up offset, stored straight to HBM.  Re-running
+//              the scans costs ALU but lets LOOK look-backs overlap;
+//   look-back: warp i handles chunks q = i (mod kNLB): aggregate publication,
+//              decoupled look-back (32 predecessors probed per round),
+//              inclusive publication, per-warp fix-up offsets.
 #pragma once
 
 #include <cuda.h>
@@ -46,10 +51,11 @@ namespace sat {
 
 enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2 };
 
-constexpr int kNCW = 8;                     // compute warps
-constexpr int kThreads = (kNCW + 2) * 32;   // + producer warp + look-back warp
+constexpr int kNCW = 8;                          // compute warps
+constexpr int kNLB = 2;                          // look-back warps
 constexpr int kProducerWarp = kNCW;
-constexpr int kLookbackWarp = kNCW + 1;
+constexpr int kFirstLbWarp = kNCW + 1;
+constexpr int kThreads = (kNCW + 1 + kNLB) * 32;
 constexpr uint32_t kFull = 0xffffffffu;
 
 // Status word: (epoch << 2) | st,  st: 0 none, 1 aggregate, 2 inclusive.
@@ -65,7 +71,8 @@ struct Cfg<P8U32S> {
   static constexpr int G = 2;   // groups per lane: cols {4l..4l+3} and {128+4l..}
   static constexpr int TW = 32 * E * G;  // 256
   static constexpr int TH = 32;
-  static constexpr int NSTAGE = 6;
+  static constexpr int LOOK = 3;         // pass B runs LOOK chunks behind pass A
+  static constexpr int NSTAGE = 8;       // LOOK + 1 resident + prefetch
 };
 template <>
 struct Cfg<P32F32F> {
@@ -75,7 +82,8 @@ struct Cfg<P32F32F> {
   static constexpr int G = 1;
   static constexpr int TW = 128;
   static constexpr int TH = 32;
-  static constexpr int NSTAGE = 4;
+  static constexpr int LOOK = 2;
+  static constexpr int NSTAGE = 6;
 };
 template <>
 struct Cfg<P64F64F> {
@@ -85,8 +93,12 @@ struct Cfg<P64F64F> {
   static constexpr int G = 1;
   static constexpr int TW = 64;
   static constexpr int TH = 32;
-  static constexpr int NSTAGE = 4;
+  static constexpr int LOOK = 2;
+  static constexpr int NSTAGE = 6;
 };
+
+template <int P>
+constexpr int kNTot = Cfg<P>::LOOK + 1;   // column-total / offset slots
 
 struct KParams {
   const char* in;       // generic-path input base (TMA path uses the tensor map)
@@ -100,24 +112,64 @@ struct KParams {
   uint32_t epoch;                        // status-word epoch of this launch
   uint64_t ticket_base;                  // counter value at launch
   unsigned long long* counter;           // ticket counter (workspace)
-  uint32_t* flags;                       // [total_bands][nchunks] status words
-  void* payload;                         // [total_bands][nchunks][2][TW] carries
+  uint32_t* flags;                       // [total_bands][nchunks] status words (hints)
+  void* payload;                         // [total_bands][nchunks][2][kVecWords] tagged carries
   const void* carry_in;                  // optional S(r0-1, .) row (W elems of TB) for band 0
+};
+
+// Optional phase profiling (debug builds with -DSAT_PROFILE): per-CTA shared
+// counters, each written by one warp's lane 0, summed into g_sat_prof at exit.
+#ifdef SAT_PROFILE
+__device__ unsigned long long g_sat_prof[16];
+__device__ __forceinline__ uint64_t gtime() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define SAT_PT(v) const uint64_t v = gtime()
+#define SAT_PADD(sm_, slot_, val_) \
+  if ((threadIdx.x & 31) == 0) atomicAdd(&(sm_).prof[slot_], (unsigned long long)(val_))
+#else
+#define SAT_PT(v)
+#define SAT_PADD(sm_, slot_, val_)
+#endif
+enum ProfSlot {
+  kPfComputeWaitFull = 0,   // warp 0: waiting for TMA data
+  kPfComputeWaitCarry = 1,  // warp 0: waiting for the look-back result
+  kPfComputeLocal = 2,      // warp 0: pass A
+  kPfComputeFixup = 3,      // warp 0: pass B (after the wait)
+  kPfLbWaitTot = 4,         // look-back warps: waiting for the column totals
+  kPfLbPublishAgg = 5,      // look-back warps: aggregate publication
+  kPfLbLookback = 6,        // look-back warps: probe + payload reads
+  kPfLbDepth = 7,           // vectors summed
+  kPfLbRetries = 8,         // probe rounds that found a missing predecessor
+  kPfLbChunks = 9,          // chunks handled
+  kPfLbRest = 10,           // offsets + inclusive publication
+  kPfProdWaitTicket = 11,   // producer: holding the next ticket back
 };
 
 template <int P>
 struct __align__(128) Smem {
   using C = Cfg<P>;
-  typename C::TA in[C::NSTAGE][C::TH][C::TW];  // TMA destination ring
-  typename C::TB tot[2][kNCW][C::TW];          // per-warp column totals -> fix-up offsets
+  typename C::TA in[C::NSTAGE][C::TH][C::TW];   // TMA destination ring
+  typename C::TB tot[kNTot<P>][kNCW][C::TW];    // per-warp column totals -> fix-up offsets
+  typename C::TB rc_in[C::NSTAGE][C::TH];       // row carries entering each resident tile
   uint64_t full[C::NSTAGE];
   uint64_t empty[C::NSTAGE];
-  uint64_t tot_full[2];
-  uint64_t carry_full[2];
-  int64_t stage_band[C::NSTAGE];
+  uint64_t tot_full[kNTot<P>];
+  uint64_t carry_full[kNTot<P>];
+  int64_t stage_band[C::NSTAGE];   // ticket (global band index), -1 = end
+  int32_t stage_img[C::NSTAGE];    // image index n
+  int32_t stage_k[C::NSTAGE];      // band index within the image
   int32_t stage_chunk[C::NSTAGE];
-  int64_t tot_band[2];
-  int32_t tot_chunk[2];
+  int64_t tot_band[kNTot<P>];
+  int32_t tot_img[kNTot<P>];
+  int32_t tot_k[kNTot<P>];
+  int32_t tot_chunk[kNTot<P>];
+  volatile uint32_t passA_done;                 // chunks through pass A (ticket pacing)
+#ifdef SAT_PROFILE
+  unsigned long long prof[16];
+#endif
 };
 
 // ---------------------------------------------------------------------------
@@ -147,13 +199,15 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 }
 
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  // try_wait with a suspend-time hint: the warp sleeps in hardware until the
+  // phase completes (or the hint expires) instead of spinning on issue slots.
   uint32_t addr = smem_u32(bar);
   asm volatile(
       "{\n\t.reg .pred p;\n\t"
       "WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
       "@!p bra WAIT_%=;\n\t}" ::"r"(addr),
-      "r"(parity)
+      "r"(parity), "r"(0x100000u)
       : "memory");
 }
 
@@ -173,30 +227,8 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
   return pol;
 }
 
-__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-
 __device__ __forceinline__ void st_relaxed_u32(uint32_t* p, uint32_t v) {
   asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// 16-byte coherent (L1-bypassing, gpu-scope relaxed) payload load.
-__device__ __forceinline__ uint4 ld_relaxed_v4(const void* p) {
-  uint4 v;
-  asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
-               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
-               : "l"(p)
-               : "memory");
-  return v;
-}
-
-__device__ __forceinline__ void st_v4(void* p, uint4 v) {
-  asm volatile("st.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
-               "r"(v.w)
-               : "memory");
 }
 
 // Streaming (evict-first) 16-byte output store.
@@ -310,140 +342,76 @@ __device__ __forceinline__ void row_step(const double* row, int lane, double& ro
   acc[0][1] += base + p1;
 }
 
-// ---------------------------------------------------------------------------
-// Compute-warp state and steps
-
+// Carry payloads are epoch-TAGGED 64-bit words: (epoch << 32) | 32 value bits
+// (an fp64 value takes two words, low then high half).  A 64-bit store is
+// single-copy atomic, so a reader that sees the current epoch in a word also
+// sees that word's value: publication needs no memory fence, and the
+// per-tile status word is only a hint telling readers which vector to read.
+// A lane's group of E elements is always 4 words (32 bytes).
 template <int P>
-struct ComputeState {
-  using C = Cfg<P>;
-  static constexpr int RW = C::TH / kNCW;
-  int s;          // input ring stage
-  uint32_t ph;    // input ring phase
-  uint32_t q;     // chunks processed by this CTA (tot/carry double-buffer index)
-  int64_t prev_band;
-  int32_t prev_chunk;
-  bool has_prev;
-  typename C::TB rowcarry[RW];
+struct Tag;
+template <>
+struct Tag<P8U32S> {
+  static __device__ __forceinline__ void enc(const uint32_t (&v)[4], uint32_t t, uint64_t (&w)[4]) {
+#pragma unroll
+    for (int e = 0; e < 4; ++e) w[e] = ((uint64_t)t << 32) | v[e];
+  }
+  static __device__ __forceinline__ void dec(const uint64_t (&w)[4], uint32_t (&v)[4]) {
+#pragma unroll
+    for (int e = 0; e < 4; ++e) v[e] = (uint32_t)w[e];
+  }
 };
-
-template <int P, bool kVecOut>
-__device__ __forceinline__ void fixup_store(Smem<P>& sm, const KParams& p,
-                                            const typename Cfg<P>::TB (&S)[Cfg<P>::TH / kNCW]
-                                                                          [Cfg<P>::G][Cfg<P>::E],
-                                            int64_t band, int32_t chunk, uint32_t q, int warp,
-                                            int lane) {
-  using C = Cfg<P>;
-  using TB = typename C::TB;
-  constexpr int RW = C::TH / kNCW;
-  const int b = q & 1;
-  mbar_wait(&sm.carry_full[b], (q >> 1) & 1);
-  TB off[C::G][C::E];
+template <>
+struct Tag<P32F32F> {
+  static __device__ __forceinline__ void enc(const float (&v)[4], uint32_t t, uint64_t (&w)[4]) {
 #pragma unroll
-  for (int g = 0; g < C::G; ++g)
-    unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[b][warp][col_of<P>(g, lane)]),
-                       off[g]);
-  const int64_t n = band / p.bands_per_image;
-  const int64_t k = band - n * p.bands_per_image;
-  char* obase = p.out + n * p.out_img_stride;
-  const int64_t x0 = (int64_t)chunk * C::TW;
+    for (int e = 0; e < 4; ++e) w[e] = ((uint64_t)t << 32) | __float_as_uint(v[e]);
+  }
+  static __device__ __forceinline__ void dec(const uint64_t (&w)[4], float (&v)[4]) {
 #pragma unroll
-  for (int i = 0; i < RW; ++i) {
-    const int64_t y = k * C::TH + warp * RW + i;
-    if (y >= p.H) break;
-    TB* orow = reinterpret_cast<TB*>(obase + y * p.out_pitch);
+    for (int e = 0; e < 4; ++e) v[e] = __uint_as_float((uint32_t)w[e]);
+  }
+};
+template <>
+struct Tag<P64F64F> {
+  static __device__ __forceinline__ void enc(const double (&v)[2], uint32_t t, uint64_t (&w)[4]) {
 #pragma unroll
-    for (int g = 0; g < C::G; ++g) {
-      const int64_t x = x0 + col_of<P>(g, lane);
-      TB v[C::E];
-#pragma unroll
-      for (int e = 0; e < C::E; ++e) v[e] = S[i][g][e] + off[g][e];
-      if (kVecOut && x + C::E <= p.W) {
-        st_cs_v4(orow + x, pack16<TB, C::E>(v));
-      } else {
-#pragma unroll
-        for (int e = 0; e < C::E; ++e)
-          if (x + e < p.W) orow[x + e] = v[e];
-      }
+    for (int e = 0; e < 2; ++e) {
+      const uint64_t b = (uint64_t)__double_as_longlong(v[e]);
+      w[2 * e] = ((uint64_t)t << 32) | (b & 0xffffffffull);
+      w[2 * e + 1] = ((uint64_t)t << 32) | (b >> 32);
     }
   }
+  static __device__ __forceinline__ void dec(const uint64_t (&w)[4], double (&v)[2]) {
+#pragma unroll
+    for (int e = 0; e < 2; ++e)
+      v[e] = __longlong_as_double((long long)((w[2 * e] & 0xffffffffull) | (w[2 * e + 1] << 32)));
+  }
+};
+
+__device__ __forceinline__ void st_relaxed_v2_u64(uint64_t* p, uint64_t a, uint64_t b) {
+  asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
 
-// One chunk of the compute warps: local pass into `cur`, then fix-up of the
-// previous chunk held in `prev`.  Returns false at the end-of-work sentinel.
-template <int P, bool kVecOut>
-__device__ __forceinline__ bool compute_step(
-    Smem<P>& sm, const KParams& p, ComputeState<P>& st,
-    typename Cfg<P>::TB (&cur)[Cfg<P>::TH / kNCW][Cfg<P>::G][Cfg<P>::E],
-    const typename Cfg<P>::TB (&prev)[Cfg<P>::TH / kNCW][Cfg<P>::G][Cfg<P>::E], int warp,
-    int lane) {
-  using C = Cfg<P>;
-  using TB = typename C::TB;
-  constexpr int RW = C::TH / kNCW;
-  mbar_wait(&sm.full[st.s], st.ph);
-  const int64_t band = sm.stage_band[st.s];
-  const int32_t chunk = sm.stage_chunk[st.s];
-  const int b = st.q & 1;
-  if (band < 0) {
-    if (st.has_prev)
-      fixup_store<P, kVecOut>(sm, p, prev, st.prev_band, st.prev_chunk, st.q - 1, warp, lane);
-    if (warp == 0 && lane == 0) sm.tot_band[b] = -1;
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&sm.tot_full[b]);
-    return false;
-  }
-  if (chunk == 0) {
-#pragma unroll
-    for (int i = 0; i < RW; ++i) st.rowcarry[i] = TB(0);
-  }
-  const typename C::TA* tile = &sm.in[st.s][warp * RW][0];
-  TB acc[C::G][C::E];
-#pragma unroll
-  for (int g = 0; g < C::G; ++g)
-#pragma unroll
-    for (int e = 0; e < C::E; ++e) acc[g][e] = TB(0);
-#pragma unroll
-  for (int i = 0; i < RW; ++i) {
-    row_step(tile + i * C::TW, lane, st.rowcarry[i], acc);
-#pragma unroll
-    for (int g = 0; g < C::G; ++g)
-#pragma unroll
-      for (int e = 0; e < C::E; ++e) cur[i][g][e] = acc[g][e];
-  }
-  __syncwarp();
-  if (lane == 0) mbar_arrive(&sm.empty[st.s]);
-  if (++st.s == C::NSTAGE) {
-    st.s = 0;
-    st.ph ^= 1u;
-  }
-  // a4: this warp's column totals for the block partial-sum scan.
-#pragma unroll
-  for (int g = 0; g < C::G; ++g)
-    *reinterpret_cast<uint4*>(&sm.tot[b][warp][col_of<P>(g, lane)]) =
-        pack16<TB, C::E>(acc[g]);
-  if (warp == 0 && lane == 0) {
-    sm.tot_band[b] = band;
-    sm.tot_chunk[b] = chunk;
-  }
-  __syncwarp();
-  if (lane == 0) mbar_arrive(&sm.tot_full[b]);
-  if (st.has_prev)
-    fixup_store<P, kVecOut>(sm, p, prev, st.prev_band, st.prev_chunk, st.q - 1, warp, lane);
-  st.has_prev = true;
-  st.prev_band = band;
-  st.prev_chunk = chunk;
-  st.q++;
-  return true;
+__device__ __forceinline__ void ld_relaxed_v2_u64(const uint64_t* p, uint64_t& a, uint64_t& b) {
+  asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
 
-// ---------------------------------------------------------------------------
-// Look-back warp
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Words of one payload vector: TW elements * (4 / E) words per element.
+template <int P>
+constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
 
 template <int P>
-__device__ __forceinline__ typename Cfg<P>::TB* payload_row(const KParams& p, int64_t band,
-                                                            int32_t chunk, int kind) {
-  using C = Cfg<P>;
-  return reinterpret_cast<typename C::TB*>(p.payload) +
-         (((band * p.nchunks + chunk) * 2 + kind) * C::TW);
+__device__ __forceinline__ uint64_t* payload_row(const KParams& p, int64_t band, int32_t chunk,
+                                                 int kind) {
+  return reinterpret_cast<uint64_t*>(p.payload) +
+         (((band * p.nchunks + chunk) * 2 + kind) * (int64_t)kVecWords<P>);
 }
 
 template <int P>
@@ -451,21 +419,80 @@ __device__ __forceinline__ void publish(const KParams& p, int64_t band, int32_t 
                                         const typename Cfg<P>::TB (&v)[Cfg<P>::G][Cfg<P>::E],
                                         int lane) {
   using C = Cfg<P>;
-  typename C::TB* row = payload_row<P>(p, band, chunk, kind);
+  uint64_t* row = payload_row<P>(p, band, chunk, kind);
 #pragma unroll
-  for (int g = 0; g < C::G; ++g) st_v4(row + col_of<P>(g, lane), pack16<typename C::TB, C::E>(v[g]));
-  __threadfence();  // each lane orders its payload stores (gpu scope) ...
-  __syncwarp();     // ... before lane 0 raises the status word
-  if (lane == 0)
+  for (int g = 0; g < C::G; ++g) {
+    uint64_t w[4];
+    Tag<P>::enc(v[g], p.epoch, w);
+    uint64_t* dst = row + (g * 32 + lane) * 4;
+    st_relaxed_v2_u64(dst, w[0], w[1]);
+    st_relaxed_v2_u64(dst + 2, w[2], w[3]);
+  }
+  __syncwarp();
+  if (lane == 0)  // hint only: readers validate every payload word's tag
     st_relaxed_u32(p.flags + band * p.nchunks + chunk,
                    (p.epoch << 2) | (kind == 0 ? kStAgg : kStIncl));
 }
 
+// Sum published vectors d = 0..dmax of the window (band j - d; kind AGG for
+// d < kk, INCL for d == kk) into acc.  Loads of a batch of kBatch vectors are
+// issued together (one L2 round trip per batch); a batch is re-read until
+// every word carries this launch's epoch.
+template <int P>
+constexpr int kBatch = Cfg<P>::G == 1 ? 4 : 2;
+
+template <int P>
+__device__ __forceinline__ void read_window(const KParams& p, int64_t j, int32_t chunk, int kk,
+                                            int dmax,
+                                            typename Cfg<P>::TB (&acc)[Cfg<P>::G][Cfg<P>::E],
+                                            int lane) {
+  using C = Cfg<P>;
+  constexpr int B = kBatch<P>;
+  for (int d0 = 0; d0 <= dmax; d0 += B) {
+    uint64_t w[B][C::G][4];
+    for (;;) {
+      bool ok = true;
+#pragma unroll
+      for (int b = 0; b < B; ++b) {
+        const int d = d0 + b;
+        if (d <= dmax) {
+          const uint64_t* row = payload_row<P>(p, j - d, chunk, d == kk ? 1 : 0);
+#pragma unroll
+          for (int g = 0; g < C::G; ++g) {
+            const uint64_t* src = row + (g * 32 + lane) * 4;
+            ld_relaxed_v2_u64(src, w[b][g][0], w[b][g][1]);
+            ld_relaxed_v2_u64(src + 2, w[b][g][2], w[b][g][3]);
+          }
+        }
+      }
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+        if (d0 + b <= dmax)
+#pragma unroll
+          for (int g = 0; g < C::G; ++g)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) ok &= (uint32_t)(w[b][g][e] >> 32) == p.epoch;
+      if (__all_sync(kFull, ok)) break;
+      __nanosleep(20);
+    }
+#pragma unroll
+    for (int b = 0; b < B; ++b)
+      if (d0 + b <= dmax)
+#pragma unroll
+        for (int g = 0; g < C::G; ++g) {
+          typename C::TB t[C::E];
+          Tag<P>::dec(w[b][g], t);
+#pragma unroll
+          for (int e = 0; e < C::E; ++e) acc[g][e] += t[e];
+        }
+  }
+}
+
 // Decoupled look-back up the tile column: V = sum of predecessors' aggregates
 // down to (and including) the nearest inclusive prefix.  32 predecessors are
-// probed per round, one per lane.
+// probed per round, one status word per lane.
 template <int P>
-__device__ __forceinline__ void lookback(const KParams& p, int64_t band, int64_t first,
+__device__ __forceinline__ void lookback(Smem<P>& sm, const KParams& p, int64_t band, int64_t first,
                                          int32_t chunk, typename Cfg<P>::TB (&V)[Cfg<P>::G][Cfg<P>::E],
                                          int lane) {
   using C = Cfg<P>;
@@ -479,7 +506,7 @@ __device__ __forceinline__ void lookback(const KParams& p, int64_t band, int64_t
     const int64_t jj = j - lane;
     uint32_t st = kStIncl;  // lanes past the image's first band: never reached
     if (jj >= first) {
-      const uint32_t f = ld_acquire_u32(p.flags + jj * p.nchunks + chunk);
+      const uint32_t f = ld_relaxed_u32(p.flags + jj * p.nchunks + chunk);
       st = ((f >> 2) == p.epoch) ? (f & 3u) : 0u;
     }
     const uint32_t inclm = __ballot_sync(kFull, st == kStIncl);
@@ -487,39 +514,35 @@ __device__ __forceinline__ void lookback(const KParams& p, int64_t band, int64_t
     const int kk = inclm ? (__ffs(inclm) - 1) : 32;
     const uint32_t need = (kk >= 31) ? kFull : ((2u << kk) - 1u);
     if (nonem & need) {
-      __nanosleep(32);
+      SAT_PADD(sm, kPfLbRetries, 1);
+      __nanosleep(20);
       continue;
     }
-    __syncwarp();
+    SAT_PADD(sm, kPfLbDepth, (kk < 32 ? kk : 31) + 1);
     const int dmax = kk < 32 ? kk : 31;
-    for (int d = 0; d <= dmax; ++d) {
-      const int kind = (d == kk) ? 1 : 0;
-      const TB* row = payload_row<P>(p, j - d, chunk, kind);
-#pragma unroll
-      for (int g = 0; g < C::G; ++g) {
-        TB t[C::E];
-        unpack16<TB, C::E>(ld_relaxed_v4(row + col_of<P>(g, lane)), t);
-#pragma unroll
-        for (int e = 0; e < C::E; ++e) V[g][e] += t[e];
-      }
-    }
+    read_window<P>(p, j, chunk, kk, dmax, V, lane);
     if (kk < 32) break;
     j -= 32;
   }
 }
 
 template <int P>
-__device__ __forceinline__ void lookback_warp(Smem<P>& sm, const KParams& p, int lane) {
+__device__ __forceinline__ void lookback_warp(Smem<P>& sm, const KParams& p, int lbw, int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
-  for (uint32_t q = 0;; ++q) {
-    const int b = q & 1;
-    mbar_wait(&sm.tot_full[b], (q >> 1) & 1);
-    const int64_t band = sm.tot_band[b];
-    const int32_t chunk = sm.tot_chunk[b];
+  constexpr int NT = kNTot<P>;
+  for (uint32_t q = lbw;; q += kNLB) {
+    const int t = q % NT;
+    SAT_PT(t0);
+    mbar_wait(&sm.tot_full[t], (q / NT) & 1);
+    SAT_PT(t1);
+    SAT_PADD(sm, kPfLbWaitTot, t1 - t0);
+    const int64_t band = sm.tot_band[t];
+    const int32_t chunk = sm.tot_chunk[t];
     if (band < 0) break;
-    const int64_t n = band / p.bands_per_image;
-    const int64_t k = band - n * p.bands_per_image;
+    SAT_PADD(sm, kPfLbChunks, 1);
+    const int64_t n = sm.tot_img[t];
+    const int64_t k = sm.tot_k[t];
     const bool has_succ = k + 1 < p.bands_per_image;
     TB V[C::G][C::E];
     if (k == 0) {
@@ -542,34 +565,184 @@ __device__ __forceinline__ void lookback_warp(Smem<P>& sm, const KParams& p, int
           for (int e = 0; e < C::E; ++e) agg[g][e] = TB(0);
 #pragma unroll
           for (int w = 0; w < kNCW; ++w) {
-            TB t[C::E];
-            unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[b][w][col_of<P>(g, lane)]),
-                               t);
+            TB tt[C::E];
+            unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]),
+                               tt);
 #pragma unroll
-            for (int e = 0; e < C::E; ++e) agg[g][e] += t[e];
+            for (int e = 0; e < C::E; ++e) agg[g][e] += tt[e];
           }
         }
         publish<P>(p, band, chunk, 0, agg, lane);
       }
-      lookback<P>(p, band, n * p.bands_per_image, chunk, V, lane);
+      SAT_PT(t2);
+      SAT_PADD(sm, kPfLbPublishAgg, t2 - t1);
+      lookback<P>(sm, p, band, n * p.bands_per_image, chunk, V, lane);
+      SAT_PT(t3);
+      SAT_PADD(sm, kPfLbLookback, t3 - t2);
     }
+    SAT_PT(t4);
     // Fix-up offsets, in place: tot[w] <- V + sum_{w' < w} tot[w'] (Fig. 3c step #2).
 #pragma unroll
     for (int g = 0; g < C::G; ++g) {
 #pragma unroll
       for (int w = 0; w < kNCW; ++w) {
-        uint4* cell = reinterpret_cast<uint4*>(&sm.tot[b][w][col_of<P>(g, lane)]);
-        TB t[C::E];
-        unpack16<TB, C::E>(*cell, t);
+        uint4* cell = reinterpret_cast<uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]);
+        TB tt[C::E];
+        unpack16<TB, C::E>(*cell, tt);
         *cell = pack16<TB, C::E>(V[g]);
 #pragma unroll
-        for (int e = 0; e < C::E; ++e) V[g][e] += t[e];
+        for (int e = 0; e < C::E; ++e) V[g][e] += tt[e];
       }
     }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sm.carry_full[t]);
     // V is now the inclusive prefix S(r1 - 1, .) of this tile column.
     if (has_succ) publish<P>(p, band, chunk, 1, V, lane);
+    SAT_PT(t5);
+    SAT_PADD(sm, kPfLbRest, t5 - t4);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Compute warps
+
+// Pass A of chunk q (stage s): row + column scans of this warp's RW rows; the
+// column totals go to tot[q % NT][warp]; the row carries entering the tile are
+// saved for pass B.  Returns false at the end-of-work sentinel.
+template <int P>
+__device__ __forceinline__ bool pass_a(Smem<P>& sm, uint32_t q, int s, uint32_t ph,
+                                       typename Cfg<P>::TB (&rowcarry)[Cfg<P>::TH / kNCW],
+                                       int warp, int lane) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  constexpr int RW = C::TH / kNCW;
+  SAT_PT(t0);
+  mbar_wait(&sm.full[s], ph);
+  SAT_PT(t1);
+  if (warp == 0) SAT_PADD(sm, kPfComputeWaitFull, t1 - t0);
+  const int64_t band = sm.stage_band[s];
+  if (band < 0) return false;
+  const int32_t chunk = sm.stage_chunk[s];
+  if (chunk == 0) {
+#pragma unroll
+    for (int i = 0; i < RW; ++i) rowcarry[i] = TB(0);
+  }
+  if (lane < RW) {
+    TB rc = rowcarry[0];
+#pragma unroll
+    for (int i = 1; i < RW; ++i)
+      if (lane == i) rc = rowcarry[i];
+    sm.rc_in[s][warp * RW + lane] = rc;
+  }
+  const typename C::TA* tile = &sm.in[s][warp * RW][0];
+  TB acc[C::G][C::E];
+#pragma unroll
+  for (int g = 0; g < C::G; ++g)
+#pragma unroll
+    for (int e = 0; e < C::E; ++e) acc[g][e] = TB(0);
+#pragma unroll
+  for (int i = 0; i < RW; ++i) row_step(tile + i * C::TW, lane, rowcarry[i], acc);
+  // a4: this warp's column totals for the block partial-sum scan.
+  const int t = q % kNTot<P>;
+#pragma unroll
+  for (int g = 0; g < C::G; ++g)
+    *reinterpret_cast<uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]) = pack16<TB, C::E>(acc[g]);
+  if (warp == 0 && lane == 0) {
+    sm.tot_band[t] = band;
+    sm.tot_img[t] = sm.stage_img[s];
+    sm.tot_k[t] = sm.stage_k[s];
+    sm.tot_chunk[t] = chunk;
+    sm.passA_done = q + 1;
+  }
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&sm.tot_full[t]);
+  SAT_PT(t2);
+  if (warp == 0) SAT_PADD(sm, kPfComputeLocal, t2 - t1);
+  return true;
+}
+
+// Pass B of chunk q (stage s): wait for the offsets, re-run the scans from the
+// resident tile, add the offsets, store; release the stage.
+template <int P, bool kVecOut>
+__device__ __forceinline__ void pass_b(Smem<P>& sm, const KParams& p, uint32_t q, int s, int warp,
+                                       int lane) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  constexpr int RW = C::TH / kNCW;
+  const int t = q % kNTot<P>;
+  SAT_PT(t0);
+  mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
+  SAT_PT(t1);
+  if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
+  TB acc[C::G][C::E];
+#pragma unroll
+  for (int g = 0; g < C::G; ++g)
+    unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]),
+                       acc[g]);
+  const int64_t n = sm.stage_img[s];
+  const int64_t k = sm.stage_k[s];
+  const int32_t chunk = sm.stage_chunk[s];
+  char* obase = p.out + n * p.out_img_stride;
+  const int64_t x0 = (int64_t)chunk * C::TW;
+  const typename C::TA* tile = &sm.in[s][warp * RW][0];
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    TB rc = sm.rc_in[s][warp * RW + i];
+    row_step(tile + i * C::TW, lane, rc, acc);  // acc = offset + S'(row i)
+    const int64_t y = k * C::TH + warp * RW + i;
+    if (y < p.H) {
+      TB* orow = reinterpret_cast<TB*>(obase + y * p.out_pitch);
+#pragma unroll
+      for (int g = 0; g < C::G; ++g) {
+        const int64_t x = x0 + col_of<P>(g, lane);
+        if (kVecOut && x + C::E <= p.W) {
+          st_cs_v4(orow + x, pack16<TB, C::E>(acc[g]));
+        } else {
+#pragma unroll
+          for (int e = 0; e < C::E; ++e)
+            if (x + e < p.W) orow[x + e] = acc[g][e];
+        }
+      }
+    }
+  }
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&sm.empty[s]);
+  SAT_PT(t2);
+  if (warp == 0) SAT_PADD(sm, kPfComputeFixup, t2 - t1);
+}
+
+template <int P, bool kVecOut>
+__device__ __forceinline__ void compute_warp(Smem<P>& sm, const KParams& p, int warp, int lane) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  constexpr int RW = C::TH / kNCW;
+  TB rowcarry[RW];
+#pragma unroll
+  for (int i = 0; i < RW; ++i) rowcarry[i] = TB(0);
+  uint32_t qa = 0, qb = 0;
+  bool ended = false;
+  for (;;) {
+    if (!ended) {
+      if (pass_a<P>(sm, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
+        ++qa;
+      else
+        ended = true;
+    }
+    if (qb < qa && (ended || qa - qb > (uint32_t)C::LOOK)) {
+      pass_b<P, kVecOut>(sm, p, qb, qb % C::NSTAGE, warp, lane);
+      ++qb;
+    } else if (ended) {
+      break;
+    }
+  }
+  // One end-of-work sentinel per look-back warp (slots are free: all pass B done).
+  for (int i = 0; i < kNLB; ++i) {
+    const uint32_t q = qa + i;
+    const int t = q % kNTot<P>;
+    if (warp == 0 && lane == 0) sm.tot_band[t] = -1;
     __syncwarp();
-    if (lane == 0) mbar_arrive(&sm.carry_full[b]);
+    if (lane == 0) mbar_arrive(&sm.tot_full[t]);
+    // the next sentinel reuses a slot only after its look-back warp left
   }
 }
 
@@ -582,11 +755,18 @@ __device__ __forceinline__ void producer_warp(Smem<P>& sm, const KParams& p, con
   using C = Cfg<P>;
   using TA = typename C::TA;
   constexpr uint32_t kTileBytes = C::TH * C::TW * sizeof(TA);
-  int s = 0;
-  uint32_t ph = 0;
+  constexpr uint32_t kTicketLead = 2;  // chunks of the current band still ahead of pass A
+  uint32_t q = 0;
   uint64_t pol = 0;
   if (kTMA) pol = policy_evict_first();
   for (;;) {
+    // Draw the next band only when pass A is within kTicketLead chunks of the
+    // end of what was issued, so a drawn band is never queued behind a whole
+    // band (its successors would stall on it).
+    SAT_PT(t0);
+    while (q > kTicketLead && sm.passA_done + kTicketLead < q) __nanosleep(64);
+    SAT_PT(t1);
+    if (lane == 0) SAT_PADD(sm, kPfProdWaitTicket, t1 - t0);
     int64_t t = 0;
     if (lane == 0) t = (int64_t)(atomicAdd(p.counter, 1ull) - p.ticket_base);
     t = __shfl_sync(kFull, t, 0);
@@ -594,8 +774,9 @@ __device__ __forceinline__ void producer_warp(Smem<P>& sm, const KParams& p, con
     const int64_t n = done ? 0 : t / p.bands_per_image;
     const int64_t k = done ? 0 : t - n * p.bands_per_image;
     const int32_t nch = done ? 1 : p.nchunks;
-    for (int32_t c = 0; c < nch; ++c) {
-      mbar_wait(&sm.empty[s], ph ^ 1u);
+    for (int32_t c = 0; c < nch; ++c, ++q) {
+      const int s = q % C::NSTAGE;
+      mbar_wait(&sm.empty[s], ((q / C::NSTAGE) & 1) ^ 1u);
       if (done) {
         if (lane == 0) {
           sm.stage_band[s] = -1;
@@ -605,6 +786,8 @@ __device__ __forceinline__ void producer_warp(Smem<P>& sm, const KParams& p, con
       } else if (kTMA) {
         if (lane == 0) {
           sm.stage_band[s] = t;
+          sm.stage_img[s] = (int32_t)n;
+          sm.stage_k[s] = (int32_t)k;
           sm.stage_chunk[s] = c;
           mbar_arrive_expect_tx(&sm.full[s], kTileBytes);
           tma_load_3d(&sm.in[s][0][0], map, &sm.full[s], c * C::TW, (int32_t)(k * C::TH),
@@ -625,15 +808,13 @@ __device__ __forceinline__ void producer_warp(Smem<P>& sm, const KParams& p, con
         __syncwarp();
         if (lane == 0) {
           sm.stage_band[s] = t;
+          sm.stage_img[s] = (int32_t)n;
+          sm.stage_k[s] = (int32_t)k;
           sm.stage_chunk[s] = c;
           mbar_arrive(&sm.full[s]);
         }
       }
       __syncwarp();
-      if (++s == C::NSTAGE) {
-        s = 0;
-        ph ^= 1u;
-      }
     }
     if (done) break;
   }
@@ -645,8 +826,6 @@ template <int P, bool kTMA, bool kVecOut>
 __global__ void __launch_bounds__(kThreads, 2)
     sat_tile_kernel(const __grid_constant__ CUtensorMap map, const KParams p) {
   using C = Cfg<P>;
-  using TB = typename C::TB;
-  constexpr int RW = C::TH / kNCW;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   Smem<P>& sm = *reinterpret_cast<Smem<P>*>(smem_raw);
   const int warp = threadIdx.x >> 5;
@@ -657,10 +836,14 @@ __global__ void __launch_bounds__(kThreads, 2)
       mbar_init(&sm.full[s], 1);
       mbar_init(&sm.empty[s], kNCW);
     }
-    for (int b = 0; b < 2; ++b) {
-      mbar_init(&sm.tot_full[b], kNCW);
-      mbar_init(&sm.carry_full[b], 1);
+    for (int t = 0; t < kNTot<P>; ++t) {
+      mbar_init(&sm.tot_full[t], kNCW);
+      mbar_init(&sm.carry_full[t], 1);
     }
+    sm.passA_done = 0;
+#ifdef SAT_PROFILE
+    for (int i = 0; i < 16; ++i) sm.prof[i] = 0;
+#endif
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     if (kTMA)
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map)) : "memory");
@@ -669,24 +852,15 @@ __global__ void __launch_bounds__(kThreads, 2)
 
   if (warp == kProducerWarp) {
     producer_warp<P, kTMA>(sm, p, &map, lane);
-  } else if (warp == kLookbackWarp) {
-    lookback_warp<P>(sm, p, lane);
+  } else if (warp >= kFirstLbWarp) {
+    lookback_warp<P>(sm, p, warp - kFirstLbWarp, lane);
   } else {
-    ComputeState<P> st;
-    st.s = 0;
-    st.ph = 0;
-    st.q = 0;
-    st.prev_band = -1;
-    st.prev_chunk = 0;
-    st.has_prev = false;
-#pragma unroll
-    for (int i = 0; i < RW; ++i) st.rowcarry[i] = TB(0);
-    TB sa[RW][C::G][C::E], sb[RW][C::G][C::E];
-    for (;;) {
-      if (!compute_step<P, kVecOut>(sm, p, st, sa, sb, warp, lane)) break;
-      if (!compute_step<P, kVecOut>(sm, p, st, sb, sa, warp, lane)) break;
-    }
+    compute_warp<P, kVecOut>(sm, p, warp, lane);
   }
+#ifdef SAT_PROFILE
+  __syncthreads();
+  if (threadIdx.x < 16) atomicAdd(&g_sat_prof[threadIdx.x], sm.prof[threadIdx.x]);
+#endif
 }
 
 }  // namespace sat

@@ -111,8 +111,11 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
 
   // Epoch: status words from earlier launches carry older epochs.
   if (pl->epoch + 1 >= (1u << 30)) {
+    // status words hold 30 epoch bits and payload words 32: clear both on wrap
     cudaError_t e = cudaMemsetAsync(pl->flags, 0, pl->max_tiles * sizeof(uint32_t), stream);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(flags)");
+    if (e == cudaSuccess)
+      e = cudaMemsetAsync(pl->payload, 0, pl->ws_bytes - ((char*)pl->payload - (char*)pl->ws), stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(workspace)");
     pl->epoch = 0;
   }
   kp.epoch = ++pl->epoch;
@@ -146,6 +149,25 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   }
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
+#ifdef SAT_PROFILE
+  {
+    unsigned long long prof[16];
+    cudaStreamSynchronize(stream);
+    cudaMemcpyFromSymbol(prof, g_sat_prof, sizeof(prof));
+    unsigned long long zero[16] = {};
+    cudaMemcpyToSymbol(g_sat_prof, zero, sizeof(zero));
+    const double ch = prof[kPfLbChunks] ? (double)prof[kPfLbChunks] : 1.0;
+    const double ctas = (double)grid;
+    fprintf(stderr,
+            "[libsat prof] pair=%d %lldx%lld grid=%lld chunks=%.0f | per chunk (ns): compute "
+            "wait_full %.0f wait_carry %.0f local %.0f fixup %.0f | lookback wait_tot %.0f agg %.0f "
+            "lookback %.0f rest %.0f depth %.2f retries/chunk %.2f\n",
+            P, (long long)h, (long long)w, (long long)grid, ch, prof[0] / ch, prof[1] / ch,
+            prof[2] / ch, prof[3] / ch, prof[4] / ch, prof[5] / ch, prof[6] / ch, prof[10] / ch,
+            prof[7] / ch, prof[8] / ch);
+    (void)ctas;
+  }
+#endif
   // Every CTA draws exactly one failing ticket.
   pl->ticket_base += (uint64_t)kp.total_bands + (uint64_t)grid;
   pl->launches++;
@@ -323,7 +345,8 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   const int64_t TH = tile_h(pair), TW = tile_w(pair);
   pl->max_tiles = max_batch * ((max_h + TH - 1) / TH) * ((max_w + TW - 1) / TW);
   const size_t flags_bytes = ((size_t)pl->max_tiles * 4 + 255) / 256 * 256;
-  const size_t payload_bytes = (size_t)pl->max_tiles * 2 * TW * out_size(pair);
+  // two tagged vectors (aggregate, inclusive) of TW elements, 8 bytes per 32 value bits
+  const size_t payload_bytes = (size_t)pl->max_tiles * 2 * TW * (out_size(pair) / 4) * 8;
   pl->ws_bytes = 256 + flags_bytes + payload_bytes;
   sat_status st = configure(pl);
   if (st == SAT_OK) {
@@ -331,7 +354,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
     if (e != cudaSuccess) st = cuda_fail(e, "cudaMalloc(workspace)");
   }
   if (st == SAT_OK) {
-    e = cudaMemset(pl->ws, 0, 256 + flags_bytes);
+    e = cudaMemset(pl->ws, 0, pl->ws_bytes);
     if (e != cudaSuccess) st = cuda_fail(e, "cudaMemset(workspace)");
   }
   if (st != SAT_OK) {

@@ -1,0 +1,20 @@
+"""Run a single SAT config a few times (for ncu captures)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch
+
+import paper_conf_cluster_chenwttm18_b200 as sat
+import satgen
+
+pair, H, W, N, reps = (int(v) for v in sys.argv[1:6])
+dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64}[pair]
+shape = (N, H, W) if N > 1 else (H, W)
+x = torch.empty(shape, dtype=dt, device="cuda")
+satgen.fill_device(x, seed=1)
+y = torch.empty(shape, dtype=sat.out_dtype(pair), device="cuda")
+for _ in range(reps):
+    sat.sat(x, out=y)
+torch.cuda.synchronize()
