@@ -52,7 +52,10 @@ namespace sat {
 enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2 };
 
 constexpr int kNCW = 8;                          // compute warps
-constexpr int kNLB = 2;                          // look-back warps
+#ifndef SAT_NLB
+#define SAT_NLB 2
+#endif
+constexpr int kNLB = SAT_NLB;                    // look-back warps
 constexpr int kProducerWarp = kNCW;
 constexpr int kFirstLbWarp = kNCW + 1;
 constexpr int kThreads = (kNCW + 1 + kNLB) * 32;
@@ -98,7 +101,7 @@ struct Cfg<P64F64F> {
 };
 
 template <int P>
-constexpr int kNTot = Cfg<P>::LOOK + 1;   // column-total / offset slots
+constexpr int kNTot = (Cfg<P>::LOOK + 1 > kNLB) ? Cfg<P>::LOOK + 1 : kNLB;  // >= kNLB (phase safety)
 
 struct KParams {
   const char* in;       // generic-path input base (TMA path uses the tensor map)
