@@ -16,12 +16,12 @@ struct sat_plan_st {
   sat_pair pair = SAT_8U_32S;
   int64_t max_h = 0, max_w = 0, max_batch = 0;
   int num_sms = 0;
-  int ctas_per_sm[3][4] = {};  // [pair][mode: bit0 TMA, bit1 vector out]
+  int active_clusters[3][3][4] = {};  // [pair][cluster 1/4/8][mode: bit0 TMA, bit1 vec out]
+  int cluster = 4;                    // CTAs (bands) per cluster: 1, 4 or 8
   int64_t max_tiles = 0;       // capacity of the look-back workspace in tiles
   void* ws = nullptr;
   size_t ws_bytes = 0;
   unsigned long long* counter = nullptr;  // ticket counter
-  uint32_t* flags = nullptr;              // status words
   void* payload = nullptr;                // aggregate / inclusive carries
   uint32_t epoch = 0;
   uint64_t ticket_base = 0;
@@ -35,6 +35,7 @@ namespace sat {
 sat_status fail(sat_status s, const char* fmt, ...);
 sat_status cuda_fail(cudaError_t e, const char* what);
 int getenv_int(const char* name, int dflt);
+int cluster_index(int cl);
 size_t in_size(sat_pair p);
 size_t out_size(sat_pair p);
 int tile_w(sat_pair p);

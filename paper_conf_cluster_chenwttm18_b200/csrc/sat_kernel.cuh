@@ -3,7 +3,7 @@
 // What it computes: the inclusive SAT S(i,j) = sum_{y<=i, x<=j} A(y,x)
 // (Eq. 1) of pitched row-major images, in one HBM pass.
 //
-// Decomposition (SURVEY.md Sec. 8, DESIGN.md "Kernel"): the image is cut into
+// Decomposition (SURVEY.md Sec. 8, DESIGN.md Sec. 5): the image is cut into
 // row BANDS of TH rows; a band is walked left-to-right in CHUNKS of TW columns
 // by one persistent CTA.  For tile (band k, chunk c) with rows [r0, r1):
 //   R(y, x)  = rowcarry(y) + rowprefix_tile(y, x)        (horizontal carry is
@@ -12,9 +12,16 @@
 //   S'(i, x) = sum_{r0 <= y <= i} R(y, x)                (per-thread serial
 //              column scan down the tile, PAPER.md:260 ScanColumn / Alg. 2)
 //   S(i, x)  = V_up(x) + S'(i, x),  V_up(x) = S(r0 - 1, x)
-// The vertical carry V_up is the only cross-CTA quantity.  It is obtained by
-// a decoupled look-back up the tile column: each tile publishes its vertical
-// aggregate S'(r1 - 1, .) and then its inclusive prefix V_up + S'(r1 - 1, .).
+// The vertical carry V_up is the only cross-CTA quantity.  CL consecutive
+// bands form a thread-block CLUSTER (one CTA per band): their column totals
+// are combined through distributed shared memory (st.async + remote mbarrier
+// complete_tx) by the cluster's leader CTA, which alone takes part in a
+// decoupled look-back up the tile column across clusters: it publishes the
+// cluster's vertical aggregate, sums predecessors' aggregates down to the
+// nearest inclusive prefix, publishes the cluster's inclusive prefix and sends
+// every band its V_up.  The chain of concurrently active look-back
+// participants is CL times shorter than with one band per participant, and
+// the global carry traffic CL times smaller.
 //
 // Inside a tile (Alg. 2 and Alg. 3; PAPER.md:191 block
 // partial-sum scan):
@@ -24,23 +31,24 @@
 //   a5  each compute warp owns RW consecutive rows and keeps a per-thread
 //       running column sum (serial scan down the rows, Alg. 2);
 //   a4  the compute warps' column totals are combined in shared memory by
-//       the look-back warps (block partial-sum scan, Fig. 3c).
+//       the look-back warps (block partial-sum scan, Fig. 3c);
+//       the same scan over the cluster's CTAs runs in the leader.
 //
 // Warp roles (one CTA = 8 compute warps + 1 producer warp + kNLB look-back
 // warps):
-//   producer : draws band tickets (atomic counter => forward progress), late
-//              enough that a drawn band is active, and streams the band's
-//              tiles into an NSTAGE-deep shared-memory ring with TMA
-//              (cp.async.bulk.tensor.3d + mbarrier complete_tx), or with plain
-//              loads on the generic (unaligned) path;
+//   producer : the leader's producer draws cluster tickets (atomic counter =>
+//              forward progress), late enough that a drawn band is active, and
+//              hands them to the cluster's other producers through DSMEM; each
+//              producer streams its band's tiles into an NSTAGE-deep smem ring
+//              with TMA (cp.async.bulk.tensor.3d + mbarrier complete_tx), or
+//              with plain loads on the generic (unaligned) path;
 //   compute  : pass A of chunk q (row + column scans -> the warp's column
 //              totals, row carries advanced), and, LOOK chunks later, pass B
 //              of chunk q: the same scans re-run from the still-resident smem
-//              tile plus the fix-up offset, stored straight to HBM.  Re-running
-//              the scans costs ALU but lets LOOK look-backs overlap;
-//   look-back: warp i handles chunks q = i (mod kNLB): aggregate publication,
-//              decoupled look-back (32 predecessors probed per round),
-//              inclusive publication, per-warp fix-up offsets.
+//              tile plus the fix-up offset, stored straight to HBM;
+//   look-back: warp i handles chunks q = i (mod kNLB): band aggregate -> leader,
+//              (leader: cluster scan + global look-back + V_up to every band),
+//              per-warp fix-up offsets.
 #pragma once
 
 #include <cuda.h>
@@ -61,7 +69,7 @@ constexpr int kFirstLbWarp = kNCW + 1;
 constexpr int kThreads = (kNCW + 1 + kNLB) * 32;
 constexpr uint32_t kFull = 0xffffffffu;
 
-// Status word: (epoch << 2) | st,  st: 0 none, 1 aggregate, 2 inclusive.
+// Carry word tag (high 32 bits): (epoch << 2) | st,  st: 1 aggregate, 2 inclusive.
 constexpr uint32_t kStAgg = 1u, kStIncl = 2u;
 
 template <int P>
@@ -74,8 +82,8 @@ struct Cfg<P8U32S> {
   static constexpr int G = 2;   // groups per lane: cols {4l..4l+3} and {128+4l..}
   static constexpr int TW = 32 * E * G;  // 256
   static constexpr int TH = 32;
-  static constexpr int LOOK = 3;         // pass B runs LOOK chunks behind pass A
-  static constexpr int NSTAGE = 8;       // LOOK + 1 resident + prefetch
+  static constexpr int LOOK = 2;         // pass B runs LOOK chunks behind pass A
+  static constexpr int NSTAGE = 5;       // LOOK + 1 resident + prefetch
 };
 template <>
 struct Cfg<P32F32F> {
@@ -86,7 +94,7 @@ struct Cfg<P32F32F> {
   static constexpr int TW = 128;
   static constexpr int TH = 32;
   static constexpr int LOOK = 2;
-  static constexpr int NSTAGE = 6;
+  static constexpr int NSTAGE = 4;
 };
 template <>
 struct Cfg<P64F64F> {
@@ -97,8 +105,15 @@ struct Cfg<P64F64F> {
   static constexpr int TW = 64;
   static constexpr int TH = 32;
   static constexpr int LOOK = 2;
-  static constexpr int NSTAGE = 6;
+  static constexpr int NSTAGE = 4;
 };
+
+// Words of one carry payload vector: TW elements * (4 / E) 64-bit words per element.
+template <int P>
+constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
+// Payload vectors one look-back round lands in shared memory (8 KB per look-back warp).
+template <int P>
+constexpr int kLandVecs = 1024 / kVecWords<P>;
 
 template <int P>
 constexpr int kNTot = (Cfg<P>::LOOK + 1 > kNLB) ? Cfg<P>::LOOK + 1 : kNLB;  // >= kNLB (phase safety)
@@ -111,17 +126,17 @@ struct KParams {
   int64_t in_img_stride, out_img_stride; // bytes
   int64_t bands_per_image;               // ceil(H / TH)
   int64_t total_bands;                   // batch * bands_per_image
+  int64_t total_tickets;                 // ceil(total_bands / CL) cluster tickets
   int32_t nchunks;                       // ceil(W / TW)
   uint32_t epoch;                        // status-word epoch of this launch
   uint64_t ticket_base;                  // counter value at launch
   unsigned long long* counter;           // ticket counter (workspace)
-  uint32_t* flags;                       // [total_bands][nchunks] status words (hints)
-  void* payload;                         // [total_bands][nchunks][2][kVecWords] tagged carries
-  const void* carry_in;                  // optional S(r0-1, .) row (W elems of TB) for band 0
+  void* payload;                         // [tickets][nchunks][kVecWords] status-tagged carries
+  const void* carry_in;                  // optional S(r0-1, .) row (W elems of TB) for image starts
 };
 
 // Optional phase profiling (debug builds with -DSAT_PROFILE): per-CTA shared
-// counters, each written by one warp's lane 0, summed into g_sat_prof at exit.
+// counters summed into g_sat_prof at exit.
 #ifdef SAT_PROFILE
 __device__ unsigned long long g_sat_prof[16];
 __device__ __forceinline__ uint64_t gtime() {
@@ -142,27 +157,39 @@ enum ProfSlot {
   kPfComputeLocal = 2,      // warp 0: pass A
   kPfComputeFixup = 3,      // warp 0: pass B (after the wait)
   kPfLbWaitTot = 4,         // look-back warps: waiting for the column totals
-  kPfLbPublishAgg = 5,      // look-back warps: aggregate publication
-  kPfLbLookback = 6,        // look-back warps: probe + payload reads
+  kPfLbCluster = 5,         // leader: waiting for the cluster's band aggregates
+  kPfLbLookback = 6,        // leader: global probe + payload reads
   kPfLbDepth = 7,           // vectors summed
   kPfLbRetries = 8,         // probe rounds that found a missing predecessor
-  kPfLbChunks = 9,          // chunks handled
-  kPfLbRest = 10,           // offsets + inclusive publication
+  kPfLbChunks = 9,          // chunks handled (all look-back warps)
+  kPfLbWaitV = 10,          // all: waiting for V_up from the leader
   kPfProdWaitTicket = 11,   // producer: holding the next ticket back
+  kPfLeaderChunks = 12,     // chunks handled by leaders
+  kPfLbRoundTime = 13,      // leader: issue -> landed time of look-back rounds
+  kPfLbRounds = 14,         // leader: look-back rounds issued
 };
 
-template <int P>
+template <int P, int CL>
 struct __align__(128) Smem {
   using C = Cfg<P>;
   typename C::TA in[C::NSTAGE][C::TH][C::TW];   // TMA destination ring
   typename C::TB tot[kNTot<P>][kNCW][C::TW];    // per-warp column totals -> fix-up offsets
+  typename C::TB lead_in[kNTot<P>][CL][C::TW];  // leader: the cluster's band aggregates
+  typename C::TB vin[kNTot<P>][C::TW];          // V_up of this band (from the leader)
   typename C::TB rc_in[C::NSTAGE][C::TH];       // row carries entering each resident tile
+  uint64_t land[kNLB][kLandVecs<P>][kVecWords<P>];  // look-back payload landing (bulk copies)
   uint64_t full[C::NSTAGE];
   uint64_t empty[C::NSTAGE];
   uint64_t tot_full[kNTot<P>];
   uint64_t carry_full[kNTot<P>];
-  int64_t stage_band[C::NSTAGE];   // ticket (global band index), -1 = end
-  int32_t stage_img[C::NSTAGE];    // image index n
+  uint64_t lead_full[kNTot<P>];                 // tx: CL aggregates landed in lead_in
+  uint64_t vin_full[kNTot<P>];                  // tx: V_up landed in vin
+  uint64_t land_full[kNLB];                     // tx: a look-back round landed
+  uint64_t tk_full;                             // tx: ticket landed in tk_slot
+  uint64_t tk_empty;                            // leader: peers consumed the ticket
+  int64_t tk_slot;
+  int64_t stage_band[C::NSTAGE];   // global band index, -1 = end of work
+  int32_t stage_img[C::NSTAGE];    // image index n (-1: padding band of a partial cluster)
   int32_t stage_k[C::NSTAGE];      // band index within the image
   int32_t stage_chunk[C::NSTAGE];
   int64_t tot_band[kNTot<P>];
@@ -230,9 +257,6 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
   return pol;
 }
 
-__device__ __forceinline__ void st_relaxed_u32(uint32_t* p, uint32_t v) {
-  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
 
 // Streaming (evict-first) 16-byte output store.
 __device__ __forceinline__ void st_cs_v4(void* p, uint4 v) {
@@ -270,79 +294,176 @@ __device__ __forceinline__ void unpack16(uint4 r, T (&v)[E]) {
 }
 
 // ---------------------------------------------------------------------------
-// a2 + a3 + a5: scan one tile row (horizontal) and accumulate it into the
-// running column sums `acc` (vertical).  `row` points at the smem tile row.
+// Cluster / distributed-shared-memory helpers
 
-__device__ __forceinline__ void row_step(const uint8_t* row, int lane, uint32_t& rowcarry,
-                                         uint32_t (&acc)[2][4]) {
-  // a1/a2: two 4-byte groups per lane; group totals via byte dot-products.
-  const uint32_t w0 = *reinterpret_cast<const uint32_t*>(row + 4 * lane);
-  const uint32_t w1 = *reinterpret_cast<const uint32_t*>(row + 128 + 4 * lane);
-  const uint32_t t0 = __dp4a(w0, 0x01010101u, 0u);
-  const uint32_t t1 = __dp4a(w1, 0x01010101u, 0u);
-  // a3: Kogge-Stone over lanes on packed 16-bit halves (each half <= 32640).
-  const uint32_t own = t0 | (t1 << 16);
-  uint32_t inc = own;
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const uint32_t o = __shfl_up_sync(kFull, inc, d);
-    if (lane >= d) inc += o;
-  }
-  const uint32_t tot = __shfl_sync(kFull, inc, 31);
-  const uint32_t ex = inc - own;
-  const uint32_t tot0 = tot & 0xFFFFu;
-  const uint32_t base0 = rowcarry + (ex & 0xFFFFu);
-  const uint32_t base1 = rowcarry + tot0 + (ex >> 16);
-  rowcarry += tot0 + (tot >> 16);
-  // a2 + a5: in-group prefix (byte masks) + carry, accumulated down the column.
-  acc[0][0] += __dp4a(w0, 0x00000001u, base0);
-  acc[0][1] += __dp4a(w0, 0x00000101u, base0);
-  acc[0][2] += __dp4a(w0, 0x00010101u, base0);
-  acc[0][3] += __dp4a(w0, 0x01010101u, base0);
-  acc[1][0] += __dp4a(w1, 0x00000001u, base1);
-  acc[1][1] += __dp4a(w1, 0x00000101u, base1);
-  acc[1][2] += __dp4a(w1, 0x00010101u, base1);
-  acc[1][3] += __dp4a(w1, 0x01010101u, base1);
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
 }
 
-__device__ __forceinline__ void row_step(const float* row, int lane, float& rowcarry,
-                                         float (&acc)[1][4]) {
-  const float4 a = *reinterpret_cast<const float4*>(row + 4 * lane);
-  const float p0 = a.x, p1 = p0 + a.y, p2 = p1 + a.z, p3 = p2 + a.w;  // Alg. 2
-  float inc = p3;
+// Address of the same shared variable in CTA `rank` of this cluster.
+__device__ __forceinline__ uint32_t mapa(const void* local, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(smem_u32(local)), "r"(rank));
+  return r;
+}
+
+// 16-byte store into a (possibly remote) CTA's smem, completing 16 tx-bytes on
+// that CTA's mbarrier.
+__device__ __forceinline__ void st_async16(uint32_t raddr, uint4 v, uint32_t rbar) {
+  asm volatile(
+      "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
+          raddr),
+      "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(rbar)
+      : "memory");
+}
+
+__device__ __forceinline__ void st_async8(uint32_t raddr, uint64_t v, uint32_t rbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b64 [%0], %1, [%2];" ::"r"(raddr),
+               "l"(v), "r"(rbar)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t rbar) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(rbar) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
+  uint32_t addr = smem_u32(bar);
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "WAITC_%=:\n\t"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1, %2;\n\t"
+      "@!p bra WAITC_%=;\n\t}" ::"r"(addr),
+      "r"(parity), "r"(0x100000u)
+      : "memory");
+}
+
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
+                   : "memory");
+}
+
+// ---------------------------------------------------------------------------
+// a2 + a3: scan the RW rows a warp owns, all rows advancing through the
+// Kogge-Stone stages together (RW-way ILP on the shuffle latency).  Produces
+// R[i] = rowcarry_i + (in-row prefix), the row-prefixed values of row i for
+// this lane's columns, and advances the row carries.  `tile` points at the
+// warp's first smem row; rows are TW elements apart.
+
+template <int RW>
+__device__ __forceinline__ void rows_scan(const uint8_t* tile, int lane, uint32_t (&rowcarry)[RW],
+                                          uint32_t (&R)[RW][2][4]) {
+  constexpr int TW = 256;
+  uint32_t w0[RW], w1[RW], own[RW], inc[RW];
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    w0[i] = *reinterpret_cast<const uint32_t*>(tile + i * TW + 4 * lane);
+    w1[i] = *reinterpret_cast<const uint32_t*>(tile + i * TW + 128 + 4 * lane);
+  }
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    // a2: group totals by byte dot-products; two groups packed as 16-bit
+    // halves (each prefix <= 32640, no carry between halves).
+    own[i] = __dp4a(w0[i], 0x01010101u, 0u) | (__dp4a(w1[i], 0x01010101u, 0u) << 16);
+    inc[i] = own[i];
+  }
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {  // a3: Alg. 3, lane >= d (reading R10)
+    uint32_t o[RW];
+#pragma unroll
+    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+      if (lane >= d) inc[i] += o[i];
+  }
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const uint32_t tot = __shfl_sync(kFull, inc[i], 31);
+    const uint32_t ex = inc[i] - own[i];
+    const uint32_t tot0 = tot & 0xFFFFu;
+    const uint32_t base0 = rowcarry[i] + (ex & 0xFFFFu);
+    const uint32_t base1 = rowcarry[i] + tot0 + (ex >> 16);
+    rowcarry[i] += tot0 + (tot >> 16);
+    // in-group prefixes + carry: dp4a with byte masks (Alg. 2 on 4 elements)
+    R[i][0][0] = __dp4a(w0[i], 0x00000001u, base0);
+    R[i][0][1] = __dp4a(w0[i], 0x00000101u, base0);
+    R[i][0][2] = __dp4a(w0[i], 0x00010101u, base0);
+    R[i][0][3] = __dp4a(w0[i], 0x01010101u, base0);
+    R[i][1][0] = __dp4a(w1[i], 0x00000001u, base1);
+    R[i][1][1] = __dp4a(w1[i], 0x00000101u, base1);
+    R[i][1][2] = __dp4a(w1[i], 0x00010101u, base1);
+    R[i][1][3] = __dp4a(w1[i], 0x01010101u, base1);
+  }
+}
+
+template <int RW>
+__device__ __forceinline__ void rows_scan(const float* tile, int lane, float (&rowcarry)[RW],
+                                          float (&R)[RW][1][4]) {
+  constexpr int TW = 128;
+  float p[RW][4], inc[RW];
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const float4 a = *reinterpret_cast<const float4*>(tile + i * TW + 4 * lane);
+    p[i][0] = a.x;  // Alg. 2
+    p[i][1] = p[i][0] + a.y;
+    p[i][2] = p[i][1] + a.z;
+    p[i][3] = p[i][2] + a.w;
+    inc[i] = p[i][3];
+  }
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {  // Alg. 3
-    const float o = __shfl_up_sync(kFull, inc, d);
-    if (lane >= d) inc += o;
+    float o[RW];
+#pragma unroll
+    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+      if (lane >= d) inc[i] += o[i];
   }
-  const float tot = __shfl_sync(kFull, inc, 31);
-  float ex = __shfl_up_sync(kFull, inc, 1);
-  if (lane == 0) ex = 0.0f;
-  const float base = rowcarry + ex;
-  rowcarry += tot;
-  acc[0][0] += base + p0;
-  acc[0][1] += base + p1;
-  acc[0][2] += base + p2;
-  acc[0][3] += base + p3;
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const float tot = __shfl_sync(kFull, inc[i], 31);
+    float ex = __shfl_up_sync(kFull, inc[i], 1);
+    if (lane == 0) ex = 0.0f;
+    const float base = rowcarry[i] + ex;
+    rowcarry[i] += tot;
+#pragma unroll
+    for (int e = 0; e < 4; ++e) R[i][0][e] = base + p[i][e];
+  }
 }
 
-__device__ __forceinline__ void row_step(const double* row, int lane, double& rowcarry,
-                                         double (&acc)[1][2]) {
-  const double2 a = *reinterpret_cast<const double2*>(row + 2 * lane);
-  const double p0 = a.x, p1 = p0 + a.y;
-  double inc = p1;
+template <int RW>
+__device__ __forceinline__ void rows_scan(const double* tile, int lane, double (&rowcarry)[RW],
+                                          double (&R)[RW][1][2]) {
+  constexpr int TW = 64;
+  double p[RW][2], inc[RW];
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const double2 a = *reinterpret_cast<const double2*>(tile + i * TW + 2 * lane);
+    p[i][0] = a.x;
+    p[i][1] = a.x + a.y;
+    inc[i] = p[i][1];
+  }
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
-    const double o = __shfl_up_sync(kFull, inc, d);
-    if (lane >= d) inc += o;
+    double o[RW];
+#pragma unroll
+    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+      if (lane >= d) inc[i] += o[i];
   }
-  const double tot = __shfl_sync(kFull, inc, 31);
-  double ex = __shfl_up_sync(kFull, inc, 1);
-  if (lane == 0) ex = 0.0;
-  const double base = rowcarry + ex;
-  rowcarry += tot;
-  acc[0][0] += base + p0;
-  acc[0][1] += base + p1;
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const double tot = __shfl_sync(kFull, inc[i], 31);
+    double ex = __shfl_up_sync(kFull, inc[i], 1);
+    if (lane == 0) ex = 0.0;
+    const double base = rowcarry[i] + ex;
+    rowcarry[i] += tot;
+    R[i][0][0] = base + p[i][0];
+    R[i][0][1] = base + p[i][1];
+  }
 }
 
 // Carry payloads are epoch-TAGGED 64-bit words: (epoch << 32) | 32 value bits
@@ -400,140 +521,266 @@ __device__ __forceinline__ void ld_relaxed_v2_u64(const uint64_t* p, uint64_t& a
   asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
 
-__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
+
+
+template <int P>
+__device__ __forceinline__ uint64_t* payload_row(const KParams& p, int64_t T, int32_t chunk) {
+  return reinterpret_cast<uint64_t*>(p.payload) + ((T * p.nchunks + chunk) * (int64_t)kVecWords<P>);
 }
 
-// Words of one payload vector: TW elements * (4 / E) words per element.
+// Status-tagged words: high 32 bits = (epoch << 2) | st, st = kStAgg or kStIncl.
+// One vector per (cluster ticket, chunk): written first as the aggregate, then
+// overwritten in place by the inclusive prefix.  A reader classifies a vector
+// by its words' tags (all AGG, all INCL, or not ready / mixed -> re-read).
 template <int P>
-constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
-
-template <int P>
-__device__ __forceinline__ uint64_t* payload_row(const KParams& p, int64_t band, int32_t chunk,
-                                                 int kind) {
-  return reinterpret_cast<uint64_t*>(p.payload) +
-         (((band * p.nchunks + chunk) * 2 + kind) * (int64_t)kVecWords<P>);
-}
-
-template <int P>
-__device__ __forceinline__ void publish(const KParams& p, int64_t band, int32_t chunk, int kind,
+__device__ __forceinline__ void publish(const KParams& p, int64_t T, int32_t chunk, uint32_t st,
                                         const typename Cfg<P>::TB (&v)[Cfg<P>::G][Cfg<P>::E],
                                         int lane) {
   using C = Cfg<P>;
-  uint64_t* row = payload_row<P>(p, band, chunk, kind);
+  uint64_t* row = payload_row<P>(p, T, chunk);
 #pragma unroll
   for (int g = 0; g < C::G; ++g) {
     uint64_t w[4];
-    Tag<P>::enc(v[g], p.epoch, w);
+    Tag<P>::enc(v[g], (p.epoch << 2) | st, w);
     uint64_t* dst = row + (g * 32 + lane) * 4;
     st_relaxed_v2_u64(dst, w[0], w[1]);
     st_relaxed_v2_u64(dst + 2, w[2], w[3]);
   }
-  __syncwarp();
-  if (lane == 0)  // hint only: readers validate every payload word's tag
-    st_relaxed_u32(p.flags + band * p.nchunks + chunk,
-                   (p.epoch << 2) | (kind == 0 ? kStAgg : kStIncl));
 }
 
-// Sum published vectors d = 0..dmax of the window (band j - d; kind AGG for
-// d < kk, INCL for d == kk) into acc.  Loads of a batch of kBatch vectors are
-// issued together (one L2 round trip per batch); a batch is re-read until
-// every word carries this launch's epoch.
-template <int P>
-constexpr int kBatch = Cfg<P>::G == 1 ? 4 : 2;
+// One bulk (TMA) copy global -> shared, completing `bytes` tx on a local mbarrier.
+// Bulk copies run on the TMA engine, not in the SM's LSU queue behind the
+// compute warps' output stores.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
 
-template <int P>
-__device__ __forceinline__ void read_window(const KParams& p, int64_t j, int32_t chunk, int kk,
-                                            int dmax,
-                                            typename Cfg<P>::TB (&acc)[Cfg<P>::G][Cfg<P>::E],
-                                            int lane) {
+// Decoupled look-back up the tile column over cluster tickets: V = sum of the
+// predecessors' aggregates down to (and including) the nearest inclusive
+// prefix.  Each round lands up to kLandVecs predecessor vectors in shared
+// memory with bulk copies (one per vector, on the TMA engine): one L2 round
+// trip per round, no separate status probe.  Vectors are classified by warp
+// votes on the word tags (each lane checks its own words).
+template <int P, class SM>
+__device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][kVecWords<P>],
+                                         uint64_t* land_bar, uint32_t& land_ph, const KParams& p,
+                                         int64_t T, int64_t first, int32_t chunk,
+                                         typename Cfg<P>::TB (&V)[Cfg<P>::G][Cfg<P>::E],
+                                         int lane) {
+  constexpr uint32_t kVecBytes = kVecWords<P> * 8;
   using C = Cfg<P>;
-  constexpr int B = kBatch<P>;
-  for (int d0 = 0; d0 <= dmax; d0 += B) {
-    uint64_t w[B][C::G][4];
+  using TB = typename C::TB;
+  constexpr int B = kLandVecs<P>;
+  const uint32_t tag_agg = (p.epoch << 2) | kStAgg, tag_incl = (p.epoch << 2) | kStIncl;
+#pragma unroll
+  for (int g = 0; g < C::G; ++g)
+#pragma unroll
+    for (int e = 0; e < C::E; ++e) V[g][e] = TB(0);
+  int64_t j = T - 1;
+  for (;;) {
+    const int nb = (j - first + 1) < B ? (int)(j - first + 1) : B;
+    int kk = nb;  // index of the inclusive vector in this round (nb: none)
     for (;;) {
-      bool ok = true;
+      __syncwarp();  // every lane is done reading the previous round's landing zone
+      if (lane == 0) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_arrive_expect_tx(land_bar, nb * kVecBytes);
+        for (int b = 0; b < nb; ++b) bulk_g2s(&land[b][0], payload_row<P>(p, j - b, chunk), kVecBytes, land_bar);
+      }
+      SAT_PT(r0);
+      mbar_wait(land_bar, land_ph);
+      SAT_PT(r1);
+      SAT_PADD(sm, kPfLbRoundTime, r1 - r0);
+      SAT_PADD(sm, kPfLbRounds, 1);
+      land_ph ^= 1u;
+      bool ready = true;
+      kk = nb;
+      for (int b = 0; b < nb; ++b) {
+        bool all_incl = true, all_agg = true;
 #pragma unroll
-      for (int b = 0; b < B; ++b) {
-        const int d = d0 + b;
-        if (d <= dmax) {
-          const uint64_t* row = payload_row<P>(p, j - d, chunk, d == kk ? 1 : 0);
+        for (int g = 0; g < C::G; ++g)
 #pragma unroll
-          for (int g = 0; g < C::G; ++g) {
-            const uint64_t* src = row + (g * 32 + lane) * 4;
-            ld_relaxed_v2_u64(src, w[b][g][0], w[b][g][1]);
-            ld_relaxed_v2_u64(src + 2, w[b][g][2], w[b][g][3]);
+          for (int e = 0; e < 4; ++e) {
+            const uint32_t tg = (uint32_t)(land[b][(g * 32 + lane) * 4 + e] >> 32);
+            all_incl &= tg == tag_incl;
+            all_agg &= tg == tag_agg;
           }
+        if (__all_sync(kFull, all_incl)) {
+          kk = b;
+          break;
+        }
+        if (!__all_sync(kFull, all_agg)) {
+          ready = false;  // predecessor not published yet (or mid-overwrite)
+          break;
         }
       }
-#pragma unroll
-      for (int b = 0; b < B; ++b)
-        if (d0 + b <= dmax)
-#pragma unroll
-          for (int g = 0; g < C::G; ++g)
-#pragma unroll
-            for (int e = 0; e < 4; ++e) ok &= (uint32_t)(w[b][g][e] >> 32) == p.epoch;
-      if (__all_sync(kFull, ok)) break;
-      __nanosleep(20);
+      if (ready) break;
+      SAT_PADD(sm, kPfLbRetries, 1);
+      __nanosleep(32);
     }
+    const int nsum = kk < nb ? kk + 1 : nb;
+    SAT_PADD(sm, kPfLbDepth, nsum);
+    for (int b = 0; b < nsum; ++b)
 #pragma unroll
-    for (int b = 0; b < B; ++b)
-      if (d0 + b <= dmax)
+      for (int g = 0; g < C::G; ++g) {
+        uint64_t w[4];
 #pragma unroll
-        for (int g = 0; g < C::G; ++g) {
-          typename C::TB t[C::E];
-          Tag<P>::dec(w[b][g], t);
+        for (int e = 0; e < 4; ++e) w[e] = land[b][(g * 32 + lane) * 4 + e];
+        TB t[C::E];
+        Tag<P>::dec(w, t);
 #pragma unroll
-          for (int e = 0; e < C::E; ++e) acc[g][e] += t[e];
-        }
+        for (int e = 0; e < C::E; ++e) V[g][e] += t[e];
+      }
+    if (kk < nb) break;
+    j -= nb;
   }
 }
 
-// Decoupled look-back up the tile column: V = sum of predecessors' aggregates
-// down to (and including) the nearest inclusive prefix.  32 predecessors are
-// probed per round, one status word per lane.
 template <int P>
-__device__ __forceinline__ void lookback(Smem<P>& sm, const KParams& p, int64_t band, int64_t first,
-                                         int32_t chunk, typename Cfg<P>::TB (&V)[Cfg<P>::G][Cfg<P>::E],
-                                         int lane) {
+__device__ __forceinline__ void load_carry_in(const KParams& p, int32_t chunk,
+                                              typename Cfg<P>::TB (&V)[Cfg<P>::G][Cfg<P>::E],
+                                              int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
 #pragma unroll
   for (int g = 0; g < C::G; ++g)
 #pragma unroll
-    for (int e = 0; e < C::E; ++e) V[g][e] = TB(0);
-  int64_t j = band - 1;
-  for (;;) {
-    const int64_t jj = j - lane;
-    uint32_t st = kStIncl;  // lanes past the image's first band: never reached
-    if (jj >= first) {
-      const uint32_t f = ld_relaxed_u32(p.flags + jj * p.nchunks + chunk);
-      st = ((f >> 2) == p.epoch) ? (f & 3u) : 0u;
+    for (int e = 0; e < C::E; ++e) {
+      const int64_t x = (int64_t)chunk * C::TW + col_of<P>(g, lane) + e;
+      V[g][e] = (p.carry_in != nullptr && x < p.W) ? reinterpret_cast<const TB*>(p.carry_in)[x]
+                                                   : TB(0);
     }
-    const uint32_t inclm = __ballot_sync(kFull, st == kStIncl);
-    const uint32_t nonem = __ballot_sync(kFull, st == 0u);
-    const int kk = inclm ? (__ffs(inclm) - 1) : 32;
-    const uint32_t need = (kk >= 31) ? kFull : ((2u << kk) - 1u);
-    if (nonem & need) {
-      SAT_PADD(sm, kPfLbRetries, 1);
-      __nanosleep(20);
-      continue;
-    }
-    SAT_PADD(sm, kPfLbDepth, (kk < 32 ? kk : 31) + 1);
-    const int dmax = kk < 32 ? kk : 31;
-    read_window<P>(p, j, chunk, kk, dmax, V, lane);
-    if (kk < 32) break;
-    j -= 32;
-  }
 }
 
-template <int P>
-__device__ __forceinline__ void lookback_warp(Smem<P>& sm, const KParams& p, int lbw, int lane) {
+// Leader CTA, chunk q (slot t): wait for the cluster's CL band aggregates,
+// publish / look back for the cluster, and send every band of the cluster its
+// V_up (segmented at image starts inside the cluster).
+template <int P, int CL>
+__device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, int lbw,
+                                             uint32_t& land_ph, int t, uint32_t q,
+                                             int64_t g0, int32_t n0, int32_t k0, int32_t chunk,
+                                             int lane) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  constexpr uint32_t kVecBytes = C::TW * sizeof(TB);
+  SAT_PT(t0);
+  mbar_wait_cluster(&sm.lead_full[t], (q / kNTot<P>) & 1);
+  SAT_PT(t1);
+  SAT_PADD(sm, kPfLbCluster, t1 - t0);
+  SAT_PADD(sm, kPfLeaderChunks, 1);
+  const int64_t T = g0 / CL;
+  const int64_t bpi = p.bands_per_image;
+  // Pass 1: the tail segment (bands of the cluster's last image) and its sum.
+  TB tail[C::G][C::E];
+  bool tail_self = (k0 == 0);
+  int64_t tail_last_k = k0;
+  {
+    int64_t k = k0;
+#pragma unroll
+    for (int g = 0; g < C::G; ++g)
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) tail[g][e] = TB(0);
+    for (int r = 0; r < CL; ++r) {
+      if (g0 + r >= p.total_bands) break;
+      if (r > 0 && k == 0) {
+        tail_self = true;
+#pragma unroll
+        for (int g = 0; g < C::G; ++g)
+#pragma unroll
+          for (int e = 0; e < C::E; ++e) tail[g][e] = TB(0);
+      }
+#pragma unroll
+      for (int g = 0; g < C::G; ++g) {
+        TB a[C::E];
+        unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.lead_in[t][r][col_of<P>(g, lane)]), a);
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) tail[g][e] += a[e];
+      }
+      tail_last_k = k;
+      if (++k == bpi) k = 0;
+    }
+  }
+  const bool has_succ = tail_last_k + 1 < bpi;
+  const bool head_self = (k0 == 0);
+  TB carry0[C::G][C::E];
+  load_carry_in<P>(p, chunk, carry0, lane);
+  if (has_succ) {
+    if (tail_self) {
+      TB incl[C::G][C::E];
+#pragma unroll
+      for (int g = 0; g < C::G; ++g)
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) incl[g][e] = carry0[g][e] + tail[g][e];
+      publish<P>(p, T, chunk, kStIncl, incl, lane);
+    } else {
+      publish<P>(p, T, chunk, kStAgg, tail, lane);
+    }
+  }
+  TB Vcl[C::G][C::E];
+  if (!head_self) {
+    SAT_PT(t2);
+    const int64_t first = ((int64_t)n0 * bpi) / CL;
+    lookback<P>(sm, sm.land[lbw], &sm.land_full[lbw], land_ph, p, T, first, chunk, Vcl, lane);
+    SAT_PT(t3);
+    SAT_PADD(sm, kPfLbLookback, t3 - t2);
+  }
+  // Pass 2: V_up of every band of the cluster (padding CTAs get zeros).
+  {
+    TB run[C::G][C::E];
+#pragma unroll
+    for (int g = 0; g < C::G; ++g)
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) run[g][e] = head_self ? carry0[g][e] : Vcl[g][e];
+    int64_t k = k0;
+    for (int r = 0; r < CL; ++r) {
+      const bool valid = g0 + r < p.total_bands;
+      if (valid && r > 0 && k == 0) {
+#pragma unroll
+        for (int g = 0; g < C::G; ++g)
+#pragma unroll
+          for (int e = 0; e < C::E; ++e) run[g][e] = carry0[g][e];
+      }
+      const uint32_t rbar = mapa(&sm.vin_full[t], r);
+#pragma unroll
+      for (int g = 0; g < C::G; ++g) {
+        TB v[C::E], a[C::E];
+        // read this band's aggregate BEFORE sending it its V_up: once CTA r has
+        // its V_up it may eventually overwrite lead_in[t][r] for chunk q + NT
+        unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.lead_in[t][r][col_of<P>(g, lane)]),
+                           a);
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) {
+          v[e] = valid ? run[g][e] : TB(0);
+          if (valid) run[g][e] += a[e];
+        }
+        st_async16(mapa(&sm.vin[t][col_of<P>(g, lane)], r), pack16<TB, C::E>(v), rbar);
+      }
+      if (++k == bpi) k = 0;
+    }
+  }
+  if (has_succ && !tail_self) {
+    TB incl[C::G][C::E];
+#pragma unroll
+    for (int g = 0; g < C::G; ++g)
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) incl[g][e] = Vcl[g][e] + tail[g][e];
+    publish<P>(p, T, chunk, kStIncl, incl, lane);
+  }
+  (void)kVecBytes;
+}
+
+template <int P, int CL>
+__device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p, int lbw,
+                                              uint32_t rank, int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr int NT = kNTot<P>;
+  constexpr uint32_t kVecBytes = C::TW * sizeof(TB);
+  uint32_t land_ph = 0;
   for (uint32_t q = lbw;; q += kNLB) {
     const int t = q % NT;
     SAT_PT(t0);
@@ -541,49 +788,42 @@ __device__ __forceinline__ void lookback_warp(Smem<P>& sm, const KParams& p, int
     SAT_PT(t1);
     SAT_PADD(sm, kPfLbWaitTot, t1 - t0);
     const int64_t band = sm.tot_band[t];
-    const int32_t chunk = sm.tot_chunk[t];
     if (band < 0) break;
     SAT_PADD(sm, kPfLbChunks, 1);
-    const int64_t n = sm.tot_img[t];
-    const int64_t k = sm.tot_k[t];
-    const bool has_succ = k + 1 < p.bands_per_image;
-    TB V[C::G][C::E];
-    if (k == 0) {
-      // Image's top band: the predecessor is the (optional) carry-in row.
+    const int32_t chunk = sm.tot_chunk[t];
+    // Arm the V_up receive before our aggregate can reach the leader.
+    if (lane == 0) mbar_arrive_expect_tx(&sm.vin_full[t], kVecBytes);
+    if (rank == 0 && lane == 0) mbar_arrive_expect_tx(&sm.lead_full[t], CL * kVecBytes);
+    __syncwarp();
+    // This band's aggregate (sum of the warps' column totals) -> leader.
+    {
+      const uint32_t rbar = mapa(&sm.lead_full[t], 0);
 #pragma unroll
-      for (int g = 0; g < C::G; ++g)
+      for (int g = 0; g < C::G; ++g) {
+        TB agg[C::E];
 #pragma unroll
-        for (int e = 0; e < C::E; ++e) {
-          const int64_t x = (int64_t)chunk * C::TW + col_of<P>(g, lane) + e;
-          V[g][e] = (p.carry_in != nullptr && x < p.W)
-                        ? reinterpret_cast<const TB*>(p.carry_in)[x]
-                        : TB(0);
+        for (int e = 0; e < C::E; ++e) agg[e] = TB(0);
+#pragma unroll
+        for (int w = 0; w < kNCW; ++w) {
+          TB tt[C::E];
+          unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]), tt);
+#pragma unroll
+          for (int e = 0; e < C::E; ++e) agg[e] += tt[e];
         }
-    } else {
-      if (has_succ) {
-        TB agg[C::G][C::E];
-#pragma unroll
-        for (int g = 0; g < C::G; ++g) {
-#pragma unroll
-          for (int e = 0; e < C::E; ++e) agg[g][e] = TB(0);
-#pragma unroll
-          for (int w = 0; w < kNCW; ++w) {
-            TB tt[C::E];
-            unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]),
-                               tt);
-#pragma unroll
-            for (int e = 0; e < C::E; ++e) agg[g][e] += tt[e];
-          }
-        }
-        publish<P>(p, band, chunk, 0, agg, lane);
+        st_async16(mapa(&sm.lead_in[t][rank][col_of<P>(g, lane)], 0), pack16<TB, C::E>(agg), rbar);
       }
-      SAT_PT(t2);
-      SAT_PADD(sm, kPfLbPublishAgg, t2 - t1);
-      lookback<P>(sm, p, band, n * p.bands_per_image, chunk, V, lane);
-      SAT_PT(t3);
-      SAT_PADD(sm, kPfLbLookback, t3 - t2);
+    }
+    if (rank == 0) {
+      leader_chunk<P, CL>(sm, p, lbw, land_ph, t, q, band, sm.tot_img[t], sm.tot_k[t], chunk, lane);
     }
     SAT_PT(t4);
+    mbar_wait_cluster(&sm.vin_full[t], (q / NT) & 1);
+    SAT_PT(t5);
+    SAT_PADD(sm, kPfLbWaitV, t5 - t4);
+    TB V[C::G][C::E];
+#pragma unroll
+    for (int g = 0; g < C::G; ++g)
+      unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.vin[t][col_of<P>(g, lane)]), V[g]);
     // Fix-up offsets, in place: tot[w] <- V + sum_{w' < w} tot[w'] (Fig. 3c step #2).
 #pragma unroll
     for (int g = 0; g < C::G; ++g) {
@@ -599,10 +839,6 @@ __device__ __forceinline__ void lookback_warp(Smem<P>& sm, const KParams& p, int
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&sm.carry_full[t]);
-    // V is now the inclusive prefix S(r1 - 1, .) of this tile column.
-    if (has_succ) publish<P>(p, band, chunk, 1, V, lane);
-    SAT_PT(t5);
-    SAT_PADD(sm, kPfLbRest, t5 - t4);
   }
 }
 
@@ -612,8 +848,8 @@ __device__ __forceinline__ void lookback_warp(Smem<P>& sm, const KParams& p, int
 // Pass A of chunk q (stage s): row + column scans of this warp's RW rows; the
 // column totals go to tot[q % NT][warp]; the row carries entering the tile are
 // saved for pass B.  Returns false at the end-of-work sentinel.
-template <int P>
-__device__ __forceinline__ bool pass_a(Smem<P>& sm, uint32_t q, int s, uint32_t ph,
+template <int P, int CL>
+__device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint32_t ph,
                                        typename Cfg<P>::TB (&rowcarry)[Cfg<P>::TH / kNCW],
                                        int warp, int lane) {
   using C = Cfg<P>;
@@ -638,13 +874,18 @@ __device__ __forceinline__ bool pass_a(Smem<P>& sm, uint32_t q, int s, uint32_t 
     sm.rc_in[s][warp * RW + lane] = rc;
   }
   const typename C::TA* tile = &sm.in[s][warp * RW][0];
+  TB R[RW][C::G][C::E];
+  rows_scan<RW>(tile, lane, rowcarry, R);
+  // a5: column totals of the row-prefixed values over the warp's rows
   TB acc[C::G][C::E];
 #pragma unroll
   for (int g = 0; g < C::G; ++g)
 #pragma unroll
-    for (int e = 0; e < C::E; ++e) acc[g][e] = TB(0);
+    for (int e = 0; e < C::E; ++e) {
+      acc[g][e] = R[0][g][e];
 #pragma unroll
-  for (int i = 0; i < RW; ++i) row_step(tile + i * C::TW, lane, rowcarry[i], acc);
+      for (int i = 1; i < RW; ++i) acc[g][e] += R[i][g][e];
+    }
   // a4: this warp's column totals for the block partial-sum scan.
   const int t = q % kNTot<P>;
 #pragma unroll
@@ -666,9 +907,9 @@ __device__ __forceinline__ bool pass_a(Smem<P>& sm, uint32_t q, int s, uint32_t 
 
 // Pass B of chunk q (stage s): wait for the offsets, re-run the scans from the
 // resident tile, add the offsets, store; release the stage.
-template <int P, bool kVecOut>
-__device__ __forceinline__ void pass_b(Smem<P>& sm, const KParams& p, uint32_t q, int s, int warp,
-                                       int lane) {
+template <int P, int CL, bool kVecOut>
+__device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32_t q, int s,
+                                       int warp, int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr int RW = C::TH / kNCW;
@@ -677,33 +918,42 @@ __device__ __forceinline__ void pass_b(Smem<P>& sm, const KParams& p, uint32_t q
   mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
   SAT_PT(t1);
   if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
-  TB acc[C::G][C::E];
+  const int32_t img = sm.stage_img[s];
+  if (img >= 0) {
+    TB acc[C::G][C::E];
 #pragma unroll
-  for (int g = 0; g < C::G; ++g)
-    unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]),
-                       acc[g]);
-  const int64_t n = sm.stage_img[s];
-  const int64_t k = sm.stage_k[s];
-  const int32_t chunk = sm.stage_chunk[s];
-  char* obase = p.out + n * p.out_img_stride;
-  const int64_t x0 = (int64_t)chunk * C::TW;
-  const typename C::TA* tile = &sm.in[s][warp * RW][0];
+    for (int g = 0; g < C::G; ++g)
+      unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]),
+                         acc[g]);
+    const int64_t k = sm.stage_k[s];
+    const int32_t chunk = sm.stage_chunk[s];
+    char* obase = p.out + (int64_t)img * p.out_img_stride;
+    const int64_t x0 = (int64_t)chunk * C::TW;
+    const typename C::TA* tile = &sm.in[s][warp * RW][0];
+    TB rc[RW], R[RW][C::G][C::E];
 #pragma unroll
-  for (int i = 0; i < RW; ++i) {
-    TB rc = sm.rc_in[s][warp * RW + i];
-    row_step(tile + i * C::TW, lane, rc, acc);  // acc = offset + S'(row i)
-    const int64_t y = k * C::TH + warp * RW + i;
-    if (y < p.H) {
-      TB* orow = reinterpret_cast<TB*>(obase + y * p.out_pitch);
+    for (int i = 0; i < RW; ++i) rc[i] = sm.rc_in[s][warp * RW + i];
+    rows_scan<RW>(tile, lane, rc, R);
 #pragma unroll
-      for (int g = 0; g < C::G; ++g) {
-        const int64_t x = x0 + col_of<P>(g, lane);
-        if (kVecOut && x + C::E <= p.W) {
-          st_cs_v4(orow + x, pack16<TB, C::E>(acc[g]));
-        } else {
+    for (int i = 0; i < RW; ++i) {
+      // a5 + a8: running column sum (Alg. 2 down the rows) on top of the offset
 #pragma unroll
-          for (int e = 0; e < C::E; ++e)
-            if (x + e < p.W) orow[x + e] = acc[g][e];
+      for (int g = 0; g < C::G; ++g)
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) acc[g][e] += R[i][g][e];
+      const int64_t y = k * C::TH + warp * RW + i;
+      if (y < p.H) {
+        TB* orow = reinterpret_cast<TB*>(obase + y * p.out_pitch);
+#pragma unroll
+        for (int g = 0; g < C::G; ++g) {
+          const int64_t x = x0 + col_of<P>(g, lane);
+          if (kVecOut && x + C::E <= p.W) {
+            st_cs_v4(orow + x, pack16<TB, C::E>(acc[g]));
+          } else {
+#pragma unroll
+            for (int e = 0; e < C::E; ++e)
+              if (x + e < p.W) orow[x + e] = acc[g][e];
+          }
         }
       }
     }
@@ -714,8 +964,9 @@ __device__ __forceinline__ void pass_b(Smem<P>& sm, const KParams& p, uint32_t q
   if (warp == 0) SAT_PADD(sm, kPfComputeFixup, t2 - t1);
 }
 
-template <int P, bool kVecOut>
-__device__ __forceinline__ void compute_warp(Smem<P>& sm, const KParams& p, int warp, int lane) {
+template <int P, int CL, bool kVecOut>
+__device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, int warp,
+                                             int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr int RW = C::TH / kNCW;
@@ -726,13 +977,13 @@ __device__ __forceinline__ void compute_warp(Smem<P>& sm, const KParams& p, int 
   bool ended = false;
   for (;;) {
     if (!ended) {
-      if (pass_a<P>(sm, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
+      if (pass_a<P, CL>(sm, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
         ++qa;
       else
         ended = true;
     }
     if (qb < qa && (ended || qa - qb > (uint32_t)C::LOOK)) {
-      pass_b<P, kVecOut>(sm, p, qb, qb % C::NSTAGE, warp, lane);
+      pass_b<P, CL, kVecOut>(sm, p, qb, qb % C::NSTAGE, warp, lane);
       ++qb;
     } else if (ended) {
       break;
@@ -745,37 +996,56 @@ __device__ __forceinline__ void compute_warp(Smem<P>& sm, const KParams& p, int 
     if (warp == 0 && lane == 0) sm.tot_band[t] = -1;
     __syncwarp();
     if (lane == 0) mbar_arrive(&sm.tot_full[t]);
-    // the next sentinel reuses a slot only after its look-back warp left
   }
 }
 
 // ---------------------------------------------------------------------------
 // Producer warp
 
-template <int P, bool kTMA>
-__device__ __forceinline__ void producer_warp(Smem<P>& sm, const KParams& p, const CUtensorMap* map,
-                                              int lane) {
+template <int P, int CL, bool kTMA>
+__device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
+                                              const CUtensorMap* map, uint32_t rank, int lane) {
   using C = Cfg<P>;
   using TA = typename C::TA;
   constexpr uint32_t kTileBytes = C::TH * C::TW * sizeof(TA);
   constexpr uint32_t kTicketLead = 2;  // chunks of the current band still ahead of pass A
-  uint32_t q = 0;
+  uint32_t q = 0, draws = 0;
   uint64_t pol = 0;
   if (kTMA) pol = policy_evict_first();
   for (;;) {
-    // Draw the next band only when pass A is within kTicketLead chunks of the
-    // end of what was issued, so a drawn band is never queued behind a whole
-    // band (its successors would stall on it).
-    SAT_PT(t0);
-    while (q > kTicketLead && sm.passA_done + kTicketLead < q) __nanosleep(64);
-    SAT_PT(t1);
-    if (lane == 0) SAT_PADD(sm, kPfProdWaitTicket, t1 - t0);
-    int64_t t = 0;
-    if (lane == 0) t = (int64_t)(atomicAdd(p.counter, 1ull) - p.ticket_base);
-    t = __shfl_sync(kFull, t, 0);
-    const bool done = t >= p.total_bands;
-    const int64_t n = done ? 0 : t / p.bands_per_image;
-    const int64_t k = done ? 0 : t - n * p.bands_per_image;
+    int64_t T = 0;
+    if (rank == 0) {
+      // Draw the next cluster ticket only when pass A is within kTicketLead
+      // chunks of the end of what was issued, so a drawn band is never queued
+      // behind a whole band (its successors would stall on it).
+      SAT_PT(t0);
+      while (q > kTicketLead && sm.passA_done + kTicketLead < q) __nanosleep(64);
+      SAT_PT(t1);
+      if (lane == 0) SAT_PADD(sm, kPfProdWaitTicket, t1 - t0);
+      if (lane == 0) {
+        T = (int64_t)(atomicAdd(p.counter, 1ull) - p.ticket_base);
+        if (CL > 1) {
+          if (draws > 0) mbar_wait_cluster(&sm.tk_empty, (draws - 1) & 1);
+          for (uint32_t r = 1; r < (uint32_t)CL; ++r)
+            st_async8(mapa(&sm.tk_slot, r), (uint64_t)T, mapa(&sm.tk_full, r));
+        }
+      }
+      T = __shfl_sync(kFull, T, 0);
+    } else {
+      if (lane == 0) {
+        mbar_arrive_expect_tx(&sm.tk_full, 8);
+        mbar_wait_cluster(&sm.tk_full, draws & 1);
+        T = sm.tk_slot;
+        mbar_arrive_remote(mapa(&sm.tk_empty, 0));
+      }
+      T = __shfl_sync(kFull, T, 0);
+    }
+    ++draws;
+    const bool done = T >= p.total_tickets;
+    const int64_t g = T * CL + rank;
+    const bool valid = !done && g < p.total_bands;
+    const int64_t n = valid ? g / p.bands_per_image : 0;
+    const int64_t k = valid ? g - n * p.bands_per_image : 0;
     const int32_t nch = done ? 1 : p.nchunks;
     for (int32_t c = 0; c < nch; ++c, ++q) {
       const int s = q % C::NSTAGE;
@@ -788,30 +1058,36 @@ __device__ __forceinline__ void producer_warp(Smem<P>& sm, const KParams& p, con
         }
       } else if (kTMA) {
         if (lane == 0) {
-          sm.stage_band[s] = t;
-          sm.stage_img[s] = (int32_t)n;
+          sm.stage_band[s] = g;
+          sm.stage_img[s] = valid ? (int32_t)n : -1;
           sm.stage_k[s] = (int32_t)k;
           sm.stage_chunk[s] = c;
-          mbar_arrive_expect_tx(&sm.full[s], kTileBytes);
-          tma_load_3d(&sm.in[s][0][0], map, &sm.full[s], c * C::TW, (int32_t)(k * C::TH),
-                      (int32_t)n, pol);
+          if (valid) {
+            mbar_arrive_expect_tx(&sm.full[s], kTileBytes);
+            tma_load_3d(&sm.in[s][0][0], map, &sm.full[s], c * C::TW, (int32_t)(k * C::TH),
+                        (int32_t)n, pol);
+          } else {
+            mbar_arrive(&sm.full[s]);  // padding band: contents unused (nothing stored)
+          }
         }
       } else {
         // Generic path: plain loads, zero fill outside the image.
-        const char* ibase = p.in + n * p.in_img_stride;
-        for (int r = 0; r < C::TH; ++r) {
-          const int64_t y = k * C::TH + r;
-          for (int x = lane; x < C::TW; x += 32) {
-            const int64_t xx = (int64_t)c * C::TW + x;
-            TA v = TA(0);
-            if (y < p.H && xx < p.W) v = reinterpret_cast<const TA*>(ibase + y * p.in_pitch)[xx];
-            sm.in[s][r][x] = v;
+        if (valid) {
+          const char* ibase = p.in + n * p.in_img_stride;
+          for (int r = 0; r < C::TH; ++r) {
+            const int64_t y = k * C::TH + r;
+            for (int x = lane; x < C::TW; x += 32) {
+              const int64_t xx = (int64_t)c * C::TW + x;
+              TA v = TA(0);
+              if (y < p.H && xx < p.W) v = reinterpret_cast<const TA*>(ibase + y * p.in_pitch)[xx];
+              sm.in[s][r][x] = v;
+            }
           }
         }
         __syncwarp();
         if (lane == 0) {
-          sm.stage_band[s] = t;
-          sm.stage_img[s] = (int32_t)n;
+          sm.stage_band[s] = g;
+          sm.stage_img[s] = valid ? (int32_t)n : -1;
           sm.stage_k[s] = (int32_t)k;
           sm.stage_chunk[s] = c;
           mbar_arrive(&sm.full[s]);
@@ -825,14 +1101,15 @@ __device__ __forceinline__ void producer_warp(Smem<P>& sm, const KParams& p, con
 
 // ---------------------------------------------------------------------------
 
-template <int P, bool kTMA, bool kVecOut>
+template <int P, int CL, bool kTMA, bool kVecOut>
 __global__ void __launch_bounds__(kThreads, 2)
     sat_tile_kernel(const __grid_constant__ CUtensorMap map, const KParams p) {
   using C = Cfg<P>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  Smem<P>& sm = *reinterpret_cast<Smem<P>*>(smem_raw);
+  Smem<P, CL>& sm = *reinterpret_cast<Smem<P, CL>*>(smem_raw);
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  const uint32_t rank = CL > 1 ? cluster_rank() : 0;
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < C::NSTAGE; ++s) {
@@ -842,7 +1119,12 @@ __global__ void __launch_bounds__(kThreads, 2)
     for (int t = 0; t < kNTot<P>; ++t) {
       mbar_init(&sm.tot_full[t], kNCW);
       mbar_init(&sm.carry_full[t], 1);
+      mbar_init(&sm.lead_full[t], 1);
+      mbar_init(&sm.vin_full[t], 1);
     }
+    for (int i = 0; i < kNLB; ++i) mbar_init(&sm.land_full[i], 1);
+    mbar_init(&sm.tk_full, 1);
+    mbar_init(&sm.tk_empty, CL > 1 ? CL - 1 : 1);
     sm.passA_done = 0;
 #ifdef SAT_PROFILE
     for (int i = 0; i < 16; ++i) sm.prof[i] = 0;
@@ -851,19 +1133,25 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (kTMA)
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map)) : "memory");
   }
-  __syncthreads();
+  // Every CTA's barriers exist before any peer can signal them.
+  if (CL > 1)
+    cluster_sync_all();
+  else
+    __syncthreads();
 
   if (warp == kProducerWarp) {
-    producer_warp<P, kTMA>(sm, p, &map, lane);
+    producer_warp<P, CL, kTMA>(sm, p, &map, rank, lane);
   } else if (warp >= kFirstLbWarp) {
-    lookback_warp<P>(sm, p, warp - kFirstLbWarp, lane);
+    lookback_warp<P, CL>(sm, p, warp - kFirstLbWarp, rank, lane);
   } else {
-    compute_warp<P, kVecOut>(sm, p, warp, lane);
+    compute_warp<P, CL, kVecOut>(sm, p, warp, lane);
   }
 #ifdef SAT_PROFILE
   __syncthreads();
   if (threadIdx.x < 16) atomicAdd(&g_sat_prof[threadIdx.x], sm.prof[threadIdx.x]);
 #endif
+  // No CTA may leave while a peer can still write into its shared memory.
+  if (CL > 1) cluster_sync_all();
 }
 
 }  // namespace sat

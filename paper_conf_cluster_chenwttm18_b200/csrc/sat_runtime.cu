@@ -112,41 +112,56 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   // Epoch: status words from earlier launches carry older epochs.
   if (pl->epoch + 1 >= (1u << 30)) {
     // status words hold 30 epoch bits and payload words 32: clear both on wrap
-    cudaError_t e = cudaMemsetAsync(pl->flags, 0, pl->max_tiles * sizeof(uint32_t), stream);
-    if (e == cudaSuccess)
-      e = cudaMemsetAsync(pl->payload, 0, pl->ws_bytes - ((char*)pl->payload - (char*)pl->ws), stream);
+    cudaError_t e =
+        cudaMemsetAsync(pl->payload, 0, pl->ws_bytes - ((char*)pl->payload - (char*)pl->ws), stream);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(workspace)");
     pl->epoch = 0;
   }
   kp.epoch = ++pl->epoch;
   kp.counter = pl->counter;
-  kp.flags = pl->flags;
   kp.payload = pl->payload;
   kp.ticket_base = pl->ticket_base;
 
   const int mode = (tma ? 1 : 0) | (vec ? 2 : 0);
-  const int per_sm = pl->ctas_per_sm[P][mode];
-  int64_t grid = (int64_t)pl->num_sms * std::max(per_sm, 1);
-  const int cap = getenv_int("SAT_CTAS_PER_SM", 0);
-  if (cap > 0) grid = (int64_t)pl->num_sms * std::min(cap, std::max(per_sm, 1));
-  grid = std::min<int64_t>(grid, kp.total_bands);
-  const size_t smem = sizeof(Smem<P>);
+  int CL = pl->cluster;
+  const int cl_env = getenv_int("SAT_CLUSTER", 0);
+  if (cl_env == 1 || cl_env == 4 || cl_env == 8) CL = cl_env;
+  const int ci = cluster_index(CL);
+  kp.total_tickets = (kp.total_bands + CL - 1) / CL;
+  // Persistent grid: every co-resident cluster slot, but no more clusters than tickets.
+  int64_t clusters = std::max(pl->active_clusters[P][ci][mode], 1);
+  const int cap = getenv_int("SAT_MAX_CLUSTERS", 0);
+  if (cap > 0) clusters = std::min<int64_t>(clusters, cap);
+  clusters = std::min<int64_t>(clusters, kp.total_tickets);
+  const int64_t grid = clusters * CL;
 
-  cudaError_t e;
-  switch (mode) {
-    case 0:
-      sat_tile_kernel<P, false, false><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
-      break;
-    case 1:
-      sat_tile_kernel<P, true, false><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
-      break;
-    case 2:
-      sat_tile_kernel<P, false, true><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
-      break;
-    default:
-      sat_tile_kernel<P, true, true><<<(unsigned)grid, kThreads, smem, stream>>>(map, kp);
-      break;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)CL;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  size_t smem = 0;
+  cudaError_t e = cudaSuccess;
+#define SAT_LAUNCH_CL(CLV)                                                                  \
+  {                                                                                         \
+    smem = sizeof(Smem<P, CLV>);                                                            \
+    cfg.dynamicSmemBytes = smem;                                                            \
+    switch (mode) {                                                                         \
+      case 0: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, false, false>, map, kp); break; \
+      case 1: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, true, false>, map, kp); break;  \
+      case 2: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, false, true>, map, kp); break;  \
+      default: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, true, true>, map, kp); break;  \
+    }                                                                                       \
   }
+  if (CL == 1) SAT_LAUNCH_CL(1) else if (CL == 4) SAT_LAUNCH_CL(4) else SAT_LAUNCH_CL(8)
+#undef SAT_LAUNCH_CL
+  if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
 #ifdef SAT_PROFILE
@@ -158,22 +173,27 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
     cudaMemcpyToSymbol(g_sat_prof, zero, sizeof(zero));
     const double ch = prof[kPfLbChunks] ? (double)prof[kPfLbChunks] : 1.0;
     const double ctas = (double)grid;
+    const double lc = prof[kPfLeaderChunks] ? (double)prof[kPfLeaderChunks] : 1.0;
     fprintf(stderr,
-            "[libsat prof] pair=%d %lldx%lld grid=%lld chunks=%.0f | per chunk (ns): compute "
-            "wait_full %.0f wait_carry %.0f local %.0f fixup %.0f | lookback wait_tot %.0f agg %.0f "
-            "lookback %.0f rest %.0f depth %.2f retries/chunk %.2f\n",
-            P, (long long)h, (long long)w, (long long)grid, ch, prof[0] / ch, prof[1] / ch,
-            prof[2] / ch, prof[3] / ch, prof[4] / ch, prof[5] / ch, prof[6] / ch, prof[10] / ch,
-            prof[7] / ch, prof[8] / ch);
+            "[libsat prof] pair=%d %lldx%lld CL=%d grid=%lld chunks=%.0f | per chunk (ns): compute "
+            "wait_full %.0f wait_carry %.0f passA %.0f passB %.0f | lb wait_tot %.0f wait_V %.0f | "
+            "leader (per leader chunk): wait_cluster %.0f lookback %.0f depth %.2f retries %.2f "
+            "rounds %.2f round_ns %.0f\n",
+            P, (long long)h, (long long)w, CL, (long long)grid, ch, prof[0] / ch, prof[1] / ch,
+            prof[2] / ch, prof[3] / ch, prof[4] / ch, prof[10] / ch, prof[5] / lc, prof[6] / lc,
+            prof[7] / lc, prof[8] / lc, prof[14] / lc,
+            prof[14] ? (double)prof[13] / (double)prof[14] : 0.0);
     (void)ctas;
   }
 #endif
-  // Every CTA draws exactly one failing ticket.
-  pl->ticket_base += (uint64_t)kp.total_bands + (uint64_t)grid;
+  // Every cluster draws exactly one failing ticket.
+  pl->ticket_base += (uint64_t)kp.total_tickets + (uint64_t)clusters;
   pl->launches++;
   if (getenv_int("SAT_LOG", 0))
-    fprintf(stderr, "[libsat] pair=%d %lldx%lld batch=%lld tma=%d vec=%d grid=%lld smem=%zu epoch=%u\n",
-            P, (long long)h, (long long)w, (long long)batch, (int)tma, (int)vec, (long long)grid,
+    fprintf(stderr,
+            "[libsat] pair=%d %lldx%lld batch=%lld tma=%d vec=%d cluster=%d grid=%lld smem=%zu "
+            "epoch=%u\n",
+            P, (long long)h, (long long)w, (long long)batch, (int)tma, (int)vec, CL, (long long)grid,
             smem, kp.epoch);
   return SAT_OK;
 }
@@ -192,26 +212,47 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
 
+int cluster_index(int cl) { return cl == 1 ? 0 : (cl == 4 ? 1 : 2); }
+
 int getenv_int(const char* name, int dflt) {
   const char* v = getenv(name);
   return v && *v ? atoi(v) : dflt;
 }
 
-template <int P>
-static sat_status configure_t(sat_plan_st* pl) {
-  const size_t smem = sizeof(Smem<P>);
+template <int P, int CL>
+static sat_status configure_cl(sat_plan_st* pl) {
+  const size_t smem = sizeof(Smem<P, CL>);
   void (*fns[4])(CUtensorMap, KParams) = {
-      sat_tile_kernel<P, false, false>, sat_tile_kernel<P, true, false>,
-      sat_tile_kernel<P, false, true>, sat_tile_kernel<P, true, true>};
+      sat_tile_kernel<P, CL, false, false>, sat_tile_kernel<P, CL, true, false>,
+      sat_tile_kernel<P, CL, false, true>, sat_tile_kernel<P, CL, true, true>};
   for (int m = 0; m < 4; ++m) {
     cudaError_t e = cudaFuncSetAttribute(fns[m], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(CL * 64);
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = smem;
+    cudaLaunchAttribute attr;
+    attr.id = cudaLaunchAttributeClusterDimension;
+    attr.val.clusterDim.x = CL;
+    attr.val.clusterDim.y = 1;
+    attr.val.clusterDim.z = 1;
+    cfg.attrs = &attr;
+    cfg.numAttrs = 1;
     int n = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fns[m], kThreads, smem);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
-    pl->ctas_per_sm[P][m] = n;
+    e = cudaOccupancyMaxActiveClusters(&n, fns[m], &cfg);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
+    pl->active_clusters[P][cluster_index(CL)][m] = n;
   }
   return SAT_OK;
+}
+
+template <int P>
+static sat_status configure_t(sat_plan_st* pl) {
+  sat_status st = configure_cl<P, 1>(pl);
+  if (st == SAT_OK) st = configure_cl<P, 4>(pl);
+  if (st == SAT_OK) st = configure_cl<P, 8>(pl);
+  return st;
 }
 
 sat_status configure(sat_plan_st* pl) {
@@ -344,10 +385,10 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   pl->num_sms = prop.multiProcessorCount;
   const int64_t TH = tile_h(pair), TW = tile_w(pair);
   pl->max_tiles = max_batch * ((max_h + TH - 1) / TH) * ((max_w + TW - 1) / TW);
-  const size_t flags_bytes = ((size_t)pl->max_tiles * 4 + 255) / 256 * 256;
-  // two tagged vectors (aggregate, inclusive) of TW elements, 8 bytes per 32 value bits
-  const size_t payload_bytes = (size_t)pl->max_tiles * 2 * TW * (out_size(pair) / 4) * 8;
-  pl->ws_bytes = 256 + flags_bytes + payload_bytes;
+  // one status-tagged carry vector of TW elements per (ticket, chunk), 8 bytes per
+  // 32 value bits; tickets <= bands, so sizing by bands covers every cluster size
+  const size_t payload_bytes = (size_t)pl->max_tiles * TW * (out_size(pair) / 4) * 8;
+  pl->ws_bytes = 256 + payload_bytes;
   sat_status st = configure(pl);
   if (st == SAT_OK) {
     e = cudaMalloc(&pl->ws, pl->ws_bytes);
@@ -364,8 +405,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
     return st;
   }
   pl->counter = reinterpret_cast<unsigned long long*>(pl->ws);
-  pl->flags = reinterpret_cast<uint32_t*>(static_cast<char*>(pl->ws) + 256);
-  pl->payload = static_cast<char*>(pl->ws) + 256 + flags_bytes;
+  pl->payload = static_cast<char*>(pl->ws) + 256;
   cudaSetDevice(prev);
   *plan = pl;
   return SAT_OK;
