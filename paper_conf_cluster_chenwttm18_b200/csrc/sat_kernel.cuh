@@ -82,8 +82,8 @@ struct Cfg<P8U32S> {
   static constexpr int G = 2;   // groups per lane: cols {4l..4l+3} and {128+4l..}
   static constexpr int TW = 32 * E * G;  // 256
   static constexpr int TH = 32;
-  static constexpr int LOOK = 2;         // pass B runs LOOK chunks behind pass A
-  static constexpr int NSTAGE = 5;       // LOOK + 1 resident + prefetch
+  static constexpr int LOOK = 3;         // pass B runs LOOK chunks behind pass A
+  static constexpr int NSTAGE = 4;       // TMA prefetch depth (stages free after pass A)
 };
 template <>
 struct Cfg<P32F32F> {
@@ -93,8 +93,8 @@ struct Cfg<P32F32F> {
   static constexpr int G = 1;
   static constexpr int TW = 128;
   static constexpr int TH = 32;
-  static constexpr int LOOK = 2;
-  static constexpr int NSTAGE = 4;
+  static constexpr int LOOK = 4;
+  static constexpr int NSTAGE = 3;
 };
 template <>
 struct Cfg<P64F64F> {
@@ -104,8 +104,8 @@ struct Cfg<P64F64F> {
   static constexpr int G = 1;
   static constexpr int TW = 64;
   static constexpr int TH = 32;
-  static constexpr int LOOK = 2;
-  static constexpr int NSTAGE = 4;
+  static constexpr int LOOK = 4;
+  static constexpr int NSTAGE = 3;
 };
 
 // Words of one carry payload vector: TW elements * (4 / E) 64-bit words per element.
@@ -117,6 +117,18 @@ constexpr int kLandVecs = 1024 / kVecWords<P>;
 
 template <int P>
 constexpr int kNTot = (Cfg<P>::LOOK + 1 > kNLB) ? Cfg<P>::LOOK + 1 : kNLB;  // >= kNLB (phase safety)
+
+// Tensor memory (TMEM) holds pass A's column-scanned rows S' until pass B:
+// per warp and chunk slot, RW rows x G x E values of 32-bit words (fp64: 2 words).
+template <int P>
+constexpr int kTmemColsPerWarp =
+    (Cfg<P>::TH / kNCW) * Cfg<P>::G * Cfg<P>::E * (int)(sizeof(typename Cfg<P>::TB) / 4);
+constexpr int kTmemCols = 256;  // per CTA (2 CTAs per SM share the SM's 512 columns)
+template <int P>
+constexpr int kTmemColsPerSlot = kTmemColsPerWarp<P> * (kNCW / 4);  // 2 warps per subpartition
+static_assert(kTmemColsPerSlot<P8U32S> * kNTot<P8U32S> <= kTmemCols, "TMEM budget (8u)");
+static_assert(kTmemColsPerSlot<P32F32F> * kNTot<P32F32F> <= kTmemCols, "TMEM budget (32f)");
+static_assert(kTmemColsPerSlot<P64F64F> * kNTot<P64F64F> <= kTmemCols, "TMEM budget (64f)");
 
 struct KParams {
   const char* in;       // generic-path input base (TMA path uses the tensor map)
@@ -173,11 +185,12 @@ template <int P, int CL>
 struct __align__(128) Smem {
   using C = Cfg<P>;
   typename C::TA in[C::NSTAGE][C::TH][C::TW];   // TMA destination ring
-  typename C::TB tot[kNTot<P>][kNCW][C::TW];    // per-warp column totals -> fix-up offsets
-  typename C::TB lead_in[kNTot<P>][CL][C::TW];  // leader: the cluster's band aggregates
-  typename C::TB vin[kNTot<P>][C::TW];          // V_up of this band (from the leader)
-  typename C::TB rc_in[C::NSTAGE][C::TH];       // row carries entering each resident tile
-  uint64_t land[kNLB][kLandVecs<P>][kVecWords<P>];  // look-back payload landing (bulk copies)
+  alignas(128) typename C::TB tot[kNTot<P>][kNCW][C::TW];    // per-warp column totals -> fix-up offsets
+  alignas(128) typename C::TB lead_in[kNTot<P>][CL][C::TW];  // leader: the cluster's band aggregates
+  alignas(128) typename C::TB vin[kNTot<P>][C::TW];          // V_up of this band (from the leader)
+  int32_t meta[kNCW][kNTot<P>][4];              // per warp: (band lo, img, k, chunk) of each slot
+  uint32_t tmem_base;                           // TMEM address from tcgen05.alloc
+  alignas(128) uint64_t land[kNLB][kLandVecs<P>][kVecWords<P>];  // look-back payload landing (bulk copies)
   uint64_t full[C::NSTAGE];
   uint64_t empty[C::NSTAGE];
   uint64_t tot_full[kNTot<P>];
@@ -343,6 +356,84 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
 __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
                    : "memory");
+}
+
+// ---------------------------------------------------------------------------
+// Tensor-memory (TMEM) helpers: 32x32b shape = thread i of the warp <-> TMEM
+// lane (subpartition base + i), .xN = N consecutive 32-bit columns.
+
+__device__ __forceinline__ void tmem_st(uint32_t taddr, const uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, "
+      "%11, %12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, "
+      "%29, %30, %31, %32};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]),
+      "r"(v[8]), "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]),
+      "r"(v[16]), "r"(v[17]), "r"(v[18]), "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]),
+      "r"(v[23]), "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]), "r"(v[28]), "r"(v[29]),
+      "r"(v[30]), "r"(v[31])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st(uint32_t taddr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, "
+      "%11, %12, %13, %14, %15, %16};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]),
+      "r"(v[8]), "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, "
+      "%12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, "
+      "%30, %31}, [%32];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+        "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+        "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]),
+        "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]),
+        "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+      : "r"(taddr)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, "
+      "%12, %13, %14, %15}, [%16];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+        "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]),
+        "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() {
+  asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_wait_ld() {
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+// Pack / unpack a lane's RW x G x E values as 32-bit words for TMEM.
+__device__ __forceinline__ uint32_t w_lo(uint32_t v) { return v; }
+__device__ __forceinline__ uint32_t w_lo(float v) { return __float_as_uint(v); }
+template <typename TB, int N>
+__device__ __forceinline__ void put_words(uint32_t (&w)[N], int idx, TB v) {
+  if constexpr (sizeof(TB) == 8) {
+    const uint64_t b = (uint64_t)__double_as_longlong(v);
+    w[2 * idx] = (uint32_t)b;
+    w[2 * idx + 1] = (uint32_t)(b >> 32);
+  } else {
+    w[idx] = w_lo(v);
+  }
+}
+template <typename TB, int N>
+__device__ __forceinline__ TB get_words(const uint32_t (&w)[N], int idx) {
+  if constexpr (sizeof(TB) == 8) {
+    return __longlong_as_double((long long)(((uint64_t)w[2 * idx + 1] << 32) | w[2 * idx]));
+  } else if constexpr (sizeof(TB) == 4 && TB(0.5) != TB(0)) {
+    return __uint_as_float(w[idx]);
+  } else {
+    return (TB)w[idx];
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -845,9 +936,17 @@ __device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p,
 // ---------------------------------------------------------------------------
 // Compute warps
 
-// Pass A of chunk q (stage s): row + column scans of this warp's RW rows; the
-// column totals go to tot[q % NT][warp]; the row carries entering the tile are
-// saved for pass B.  Returns false at the end-of-work sentinel.
+// TMEM address of warp `warp`'s S' rows for chunk slot t.
+template <int P, int CL>
+__device__ __forceinline__ uint32_t tmem_addr(const Smem<P, CL>& sm, int t, int warp) {
+  return sm.tmem_base + ((uint32_t)(32 * (warp & 3)) << 16) +
+         (uint32_t)(t * kTmemColsPerSlot<P> + (warp >> 2) * kTmemColsPerWarp<P>);
+}
+
+// Pass A of chunk q (stage s): row + column scans of this warp's RW rows
+// (a2, a3, a5).  The column-scanned rows S' go to TMEM, the column totals to
+// tot[q % NT][warp]; the input stage is released at once.  Returns false at
+// the end-of-work sentinel.
 template <int P, int CL>
 __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint32_t ph,
                                        typename Cfg<P>::TB (&rowcarry)[Cfg<P>::TH / kNCW],
@@ -855,6 +954,7 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint3
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr int RW = C::TH / kNCW;
+  constexpr int NW = kTmemColsPerWarp<P>;
   SAT_PT(t0);
   mbar_wait(&sm.full[s], ph);
   SAT_PT(t1);
@@ -862,39 +962,45 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint3
   const int64_t band = sm.stage_band[s];
   if (band < 0) return false;
   const int32_t chunk = sm.stage_chunk[s];
+  const int32_t img = sm.stage_img[s];
+  const int32_t kk = sm.stage_k[s];
   if (chunk == 0) {
 #pragma unroll
     for (int i = 0; i < RW; ++i) rowcarry[i] = TB(0);
   }
-  if (lane < RW) {
-    TB rc = rowcarry[0];
-#pragma unroll
-    for (int i = 1; i < RW; ++i)
-      if (lane == i) rc = rowcarry[i];
-    sm.rc_in[s][warp * RW + lane] = rc;
-  }
   const typename C::TA* tile = &sm.in[s][warp * RW][0];
   TB R[RW][C::G][C::E];
   rows_scan<RW>(tile, lane, rowcarry, R);
-  // a5: column totals of the row-prefixed values over the warp's rows
-  TB acc[C::G][C::E];
-#pragma unroll
-  for (int g = 0; g < C::G; ++g)
-#pragma unroll
-    for (int e = 0; e < C::E; ++e) {
-      acc[g][e] = R[0][g][e];
-#pragma unroll
-      for (int i = 1; i < RW; ++i) acc[g][e] += R[i][g][e];
-    }
-  // a4: this warp's column totals for the block partial-sum scan.
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&sm.empty[s]);  // the tile is consumed: refill the stage
+  // a5: running column sums S'(row i) down the warp's rows -> TMEM
   const int t = q % kNTot<P>;
+  TB acc[C::G][C::E];
+  uint32_t w[NW];
+#pragma unroll
+  for (int i = 0; i < RW; ++i)
+#pragma unroll
+    for (int g = 0; g < C::G; ++g)
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) {
+        acc[g][e] = i == 0 ? R[0][g][e] : acc[g][e] + R[i][g][e];
+        put_words<TB>(w, (i * C::G + g) * C::E + e, acc[g][e]);
+      }
+  tmem_st(tmem_addr(sm, t, warp), w);
+  tmem_wait_st();
+  // a4: this warp's column totals for the block partial-sum scan.
 #pragma unroll
   for (int g = 0; g < C::G; ++g)
     *reinterpret_cast<uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]) = pack16<TB, C::E>(acc[g]);
+  if (lane == 0) {
+    sm.meta[warp][t][1] = img;
+    sm.meta[warp][t][2] = kk;
+    sm.meta[warp][t][3] = chunk;
+  }
   if (warp == 0 && lane == 0) {
     sm.tot_band[t] = band;
-    sm.tot_img[t] = sm.stage_img[s];
-    sm.tot_k[t] = sm.stage_k[s];
+    sm.tot_img[t] = img;
+    sm.tot_k[t] = kk;
     sm.tot_chunk[t] = chunk;
     sm.passA_done = q + 1;
   }
@@ -905,61 +1011,57 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint3
   return true;
 }
 
-// Pass B of chunk q (stage s): wait for the offsets, re-run the scans from the
-// resident tile, add the offsets, store; release the stage.
+// Pass B of chunk q: wait for the fix-up offsets, load S' back from TMEM,
+// add, store (a8).
 template <int P, int CL, bool kVecOut>
-__device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32_t q, int s,
-                                       int warp, int lane) {
+__device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32_t q, int warp,
+                                       int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr int RW = C::TH / kNCW;
+  constexpr int NW = kTmemColsPerWarp<P>;
   const int t = q % kNTot<P>;
   SAT_PT(t0);
   mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
   SAT_PT(t1);
   if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
-  const int32_t img = sm.stage_img[s];
+  const int32_t img = sm.meta[warp][t][1];
   if (img >= 0) {
-    TB acc[C::G][C::E];
+    uint32_t w[NW];
+    tmem_ld(tmem_addr(sm, t, warp), w);
+    TB off[C::G][C::E];
 #pragma unroll
     for (int g = 0; g < C::G; ++g)
       unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]),
-                         acc[g]);
-    const int64_t k = sm.stage_k[s];
-    const int32_t chunk = sm.stage_chunk[s];
+                         off[g]);
+    const int64_t k = sm.meta[warp][t][2];
+    const int32_t chunk = sm.meta[warp][t][3];
     char* obase = p.out + (int64_t)img * p.out_img_stride;
     const int64_t x0 = (int64_t)chunk * C::TW;
-    const typename C::TA* tile = &sm.in[s][warp * RW][0];
-    TB rc[RW], R[RW][C::G][C::E];
-#pragma unroll
-    for (int i = 0; i < RW; ++i) rc[i] = sm.rc_in[s][warp * RW + i];
-    rows_scan<RW>(tile, lane, rc, R);
+    tmem_wait_ld();
 #pragma unroll
     for (int i = 0; i < RW; ++i) {
-      // a5 + a8: running column sum (Alg. 2 down the rows) on top of the offset
-#pragma unroll
-      for (int g = 0; g < C::G; ++g)
-#pragma unroll
-        for (int e = 0; e < C::E; ++e) acc[g][e] += R[i][g][e];
       const int64_t y = k * C::TH + warp * RW + i;
       if (y < p.H) {
         TB* orow = reinterpret_cast<TB*>(obase + y * p.out_pitch);
 #pragma unroll
         for (int g = 0; g < C::G; ++g) {
+          TB v[C::E];
+#pragma unroll
+          for (int e = 0; e < C::E; ++e)
+            v[e] = off[g][e] + get_words<TB>(w, (i * C::G + g) * C::E + e);
           const int64_t x = x0 + col_of<P>(g, lane);
           if (kVecOut && x + C::E <= p.W) {
-            st_cs_v4(orow + x, pack16<TB, C::E>(acc[g]));
+            st_cs_v4(orow + x, pack16<TB, C::E>(v));
           } else {
 #pragma unroll
             for (int e = 0; e < C::E; ++e)
-              if (x + e < p.W) orow[x + e] = acc[g][e];
+              if (x + e < p.W) orow[x + e] = v[e];
           }
         }
       }
     }
   }
-  __syncwarp();
-  if (lane == 0) mbar_arrive(&sm.empty[s]);
   SAT_PT(t2);
   if (warp == 0) SAT_PADD(sm, kPfComputeFixup, t2 - t1);
 }
@@ -983,7 +1085,7 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
         ended = true;
     }
     if (qb < qa && (ended || qa - qb > (uint32_t)C::LOOK)) {
-      pass_b<P, CL, kVecOut>(sm, p, qb, qb % C::NSTAGE, warp, lane);
+      pass_b<P, CL, kVecOut>(sm, p, qb, warp, lane);
       ++qb;
     } else if (ended) {
       break;
@@ -1133,11 +1235,20 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (kTMA)
       asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map)) : "memory");
   }
+  if (warp == 0) {  // TMEM for the S' rows (one warp allocates and later frees)
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&sm.tmem_base)),
+                 "r"(kTmemCols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   // Every CTA's barriers exist before any peer can signal them.
   if (CL > 1)
     cluster_sync_all();
   else
     __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 
   if (warp == kProducerWarp) {
     producer_warp<P, CL, kTMA>(sm, p, &map, rank, lane);
@@ -1150,8 +1261,18 @@ __global__ void __launch_bounds__(kThreads, 2)
   __syncthreads();
   if (threadIdx.x < 16) atomicAdd(&g_sat_prof[threadIdx.x], sm.prof[threadIdx.x]);
 #endif
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   // No CTA may leave while a peer can still write into its shared memory.
-  if (CL > 1) cluster_sync_all();
+  if (CL > 1)
+    cluster_sync_all();
+  else
+    __syncthreads();
+  if (warp == 0) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(sm.tmem_base),
+                 "r"(kTmemCols)
+                 : "memory");
+  }
 }
 
 }  // namespace sat

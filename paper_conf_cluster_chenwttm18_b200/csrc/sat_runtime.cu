@@ -132,6 +132,8 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   int64_t clusters = std::max(pl->active_clusters[P][ci][mode], 1);
   const int cap = getenv_int("SAT_MAX_CLUSTERS", 0);
   if (cap > 0) clusters = std::min<int64_t>(clusters, cap);
+  const int force = getenv_int("SAT_FORCE_CLUSTERS", 0);
+  if (force > 0) clusters = force;
   clusters = std::min<int64_t>(clusters, kp.total_tickets);
   const int64_t grid = clusters * CL;
 
@@ -219,12 +221,26 @@ int getenv_int(const char* name, int dflt) {
   return v && *v ? atoi(v) : dflt;
 }
 
+// Occupancy proxy: the occupancy calculator treats any tcgen05 (TMEM) kernel as
+// one CTA per SM, while the hardware co-schedules as many as TMEM allows (each
+// CTA allocates kTmemCols of the SM's 512 columns).  The proxy has the same
+// block size, dynamic shared memory, cluster shape and register bound, so its
+// answer is the real residency, which is then capped by TMEM.
+template <int P, int CL>
+__global__ void __launch_bounds__(kThreads, 2) sat_occupancy_proxy(int* sink) {
+  extern __shared__ unsigned char s[];
+  if (sink) sink[threadIdx.x] = s[threadIdx.x];
+}
+
 template <int P, int CL>
 static sat_status configure_cl(sat_plan_st* pl) {
   const size_t smem = sizeof(Smem<P, CL>);
   void (*fns[4])(CUtensorMap, KParams) = {
       sat_tile_kernel<P, CL, false, false>, sat_tile_kernel<P, CL, true, false>,
       sat_tile_kernel<P, CL, false, true>, sat_tile_kernel<P, CL, true, true>};
+  cudaError_t e0 = cudaFuncSetAttribute(sat_occupancy_proxy<P, CL>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e0 != cudaSuccess) return cuda_fail(e0, "cudaFuncSetAttribute(proxy)");
   for (int m = 0; m < 4; ++m) {
     cudaError_t e = cudaFuncSetAttribute(fns[m], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
@@ -240,9 +256,10 @@ static sat_status configure_cl(sat_plan_st* pl) {
     cfg.attrs = &attr;
     cfg.numAttrs = 1;
     int n = 0;
-    e = cudaOccupancyMaxActiveClusters(&n, fns[m], &cfg);
+    e = cudaOccupancyMaxActiveClusters(&n, sat_occupancy_proxy<P, CL>, &cfg);
     if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
-    pl->active_clusters[P][cluster_index(CL)][m] = n;
+    const int tmem_cap = pl->num_sms * (512 / kTmemCols) / CL;
+    pl->active_clusters[P][cluster_index(CL)][m] = std::min(n, tmem_cap);
   }
   return SAT_OK;
 }
