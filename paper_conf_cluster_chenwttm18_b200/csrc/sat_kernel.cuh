@@ -61,7 +61,7 @@ enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2 };
 
 constexpr int kNCW = 8;                          // compute warps
 #ifndef SAT_NLB
-#define SAT_NLB 2
+#define SAT_NLB 3
 #endif
 constexpr int kNLB = SAT_NLB;                    // look-back warps
 constexpr int kProducerWarp = kNCW;
@@ -111,9 +111,13 @@ struct Cfg<P64F64F> {
 // Words of one carry payload vector: TW elements * (4 / E) 64-bit words per element.
 template <int P>
 constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
-// Payload vectors one look-back round lands in shared memory (8 KB per look-back warp).
+// Payload vectors one look-back round lands in shared memory (kLandWords * 8 B
+// per look-back warp).
+#ifndef SAT_LAND_WORDS
+#define SAT_LAND_WORDS 512
+#endif
 template <int P>
-constexpr int kLandVecs = 1024 / kVecWords<P>;
+constexpr int kLandVecs = (SAT_LAND_WORDS) / kVecWords<P>;
 
 template <int P>
 constexpr int kNTot = (Cfg<P>::LOOK + 1 > kNLB) ? Cfg<P>::LOOK + 1 : kNLB;  // >= kNLB (phase safety)
@@ -179,6 +183,7 @@ enum ProfSlot {
   kPfLeaderChunks = 12,     // chunks handled by leaders
   kPfLbRoundTime = 13,      // leader: issue -> landed time of look-back rounds
   kPfLbRounds = 14,         // leader: look-back rounds issued
+  kPfLbIssue = 15,          // leader: fence + bulk-copy issue time
 };
 
 template <int P, int CL>
@@ -677,12 +682,14 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
     int kk = nb;  // index of the inclusive vector in this round (nb: none)
     for (;;) {
       __syncwarp();  // every lane is done reading the previous round's landing zone
-      if (lane == 0) {
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        mbar_arrive_expect_tx(land_bar, nb * kVecBytes);
-        for (int b = 0; b < nb; ++b) bulk_g2s(&land[b][0], payload_row<P>(p, j - b, chunk), kVecBytes, land_bar);
-      }
+      SAT_PT(i0);
+      // lane b fetches vector b (parallel issue); lane 0 arms the barrier.  The
+      // previous round's generic reads of the landing zone were consumed before
+      // the __syncwarp above, so the async-proxy overwrite cannot overtake them.
+      if (lane == 0) mbar_arrive_expect_tx(land_bar, nb * kVecBytes);
+      if (lane < nb) bulk_g2s(&land[lane][0], payload_row<P>(p, j - lane, chunk), kVecBytes, land_bar);
       SAT_PT(r0);
+      SAT_PADD(sm, kPfLbIssue, r0 - i0);
       mbar_wait(land_bar, land_ph);
       SAT_PT(r1);
       SAT_PADD(sm, kPfLbRoundTime, r1 - r0);

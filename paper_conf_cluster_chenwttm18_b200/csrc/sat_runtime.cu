@@ -180,11 +180,12 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
             "[libsat prof] pair=%d %lldx%lld CL=%d grid=%lld chunks=%.0f | per chunk (ns): compute "
             "wait_full %.0f wait_carry %.0f passA %.0f passB %.0f | lb wait_tot %.0f wait_V %.0f | "
             "leader (per leader chunk): wait_cluster %.0f lookback %.0f depth %.2f retries %.2f "
-            "rounds %.2f round_ns %.0f\n",
+            "rounds %.2f round_ns %.0f issue_ns %.0f\n",
             P, (long long)h, (long long)w, CL, (long long)grid, ch, prof[0] / ch, prof[1] / ch,
             prof[2] / ch, prof[3] / ch, prof[4] / ch, prof[10] / ch, prof[5] / lc, prof[6] / lc,
             prof[7] / lc, prof[8] / lc, prof[14] / lc,
-            prof[14] ? (double)prof[13] / (double)prof[14] : 0.0);
+            prof[14] ? (double)prof[13] / (double)prof[14] : 0.0,
+            prof[14] ? (double)prof[15] / (double)prof[14] : 0.0);
     (void)ctas;
   }
 #endif
