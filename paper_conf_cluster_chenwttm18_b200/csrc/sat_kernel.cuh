@@ -186,12 +186,19 @@ enum ProfSlot {
   kPfLbIssue = 15,          // leader: fence + bulk-copy issue time
 };
 
+// Chunk q of a cluster is led by CTA q % CL (rotating leadership spreads the
+// global look-backs over all the cluster's look-back warps).  A leader's
+// gather slot is reused CL * kNLead chunks later, which must be >= kNTot so a
+// band cannot send a new aggregate into a slot its leader still reads.
+template <int P, int CL>
+constexpr int kNLead = (kNTot<P> + CL - 1) / CL;
+
 template <int P, int CL>
 struct __align__(128) Smem {
   using C = Cfg<P>;
   typename C::TA in[C::NSTAGE][C::TH][C::TW];   // TMA destination ring
   alignas(128) typename C::TB tot[kNTot<P>][kNCW][C::TW];    // per-warp column totals -> fix-up offsets
-  alignas(128) typename C::TB lead_in[kNTot<P>][CL][C::TW];  // leader: the cluster's band aggregates
+  alignas(128) typename C::TB lead_in[kNLead<P, CL>][CL][C::TW];  // chunk leader: the bands' aggregates
   alignas(128) typename C::TB vin[kNTot<P>][C::TW];          // V_up of this band (from the leader)
   int32_t meta[kNCW][kNTot<P>][4];              // per warp: (band lo, img, k, chunk) of each slot
   uint32_t tmem_base;                           // TMEM address from tcgen05.alloc
@@ -200,7 +207,7 @@ struct __align__(128) Smem {
   uint64_t empty[C::NSTAGE];
   uint64_t tot_full[kNTot<P>];
   uint64_t carry_full[kNTot<P>];
-  uint64_t lead_full[kNTot<P>];                 // tx: CL aggregates landed in lead_in
+  uint64_t lead_full[kNLead<P, CL>];            // tx: CL aggregates landed in lead_in
   uint64_t vin_full[kNTot<P>];                  // tx: V_up landed in vin
   uint64_t land_full[kNLB];                     // tx: a look-back round landed
   uint64_t tk_full;                             // tx: ticket landed in tk_slot
@@ -759,14 +766,15 @@ __device__ __forceinline__ void load_carry_in(const KParams& p, int32_t chunk,
 // V_up (segmented at image starts inside the cluster).
 template <int P, int CL>
 __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, int lbw,
-                                             uint32_t& land_ph, int t, uint32_t q,
-                                             int64_t g0, int32_t n0, int32_t k0, int32_t chunk,
-                                             int lane) {
+                                             uint32_t& land_ph, int t, int ls, uint32_t lph,
+                                             int64_t g0, int32_t chunk, int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr uint32_t kVecBytes = C::TW * sizeof(TB);
+  const int32_t n0 = (int32_t)(g0 / p.bands_per_image);
+  const int32_t k0 = (int32_t)(g0 - (int64_t)n0 * p.bands_per_image);
   SAT_PT(t0);
-  mbar_wait_cluster(&sm.lead_full[t], (q / kNTot<P>) & 1);
+  mbar_wait_cluster(&sm.lead_full[ls], lph);
   SAT_PT(t1);
   SAT_PADD(sm, kPfLbCluster, t1 - t0);
   SAT_PADD(sm, kPfLeaderChunks, 1);
@@ -794,7 +802,7 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
 #pragma unroll
       for (int g = 0; g < C::G; ++g) {
         TB a[C::E];
-        unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.lead_in[t][r][col_of<P>(g, lane)]), a);
+        unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.lead_in[ls][r][col_of<P>(g, lane)]), a);
 #pragma unroll
         for (int e = 0; e < C::E; ++e) tail[g][e] += a[e];
       }
@@ -847,8 +855,8 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
       for (int g = 0; g < C::G; ++g) {
         TB v[C::E], a[C::E];
         // read this band's aggregate BEFORE sending it its V_up: once CTA r has
-        // its V_up it may eventually overwrite lead_in[t][r] for chunk q + NT
-        unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.lead_in[t][r][col_of<P>(g, lane)]),
+        // its V_up it may eventually overwrite lead_in[ls][r] for a later chunk
+        unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.lead_in[ls][r][col_of<P>(g, lane)]),
                            a);
 #pragma unroll
         for (int e = 0; e < C::E; ++e) {
@@ -889,13 +897,18 @@ __device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p,
     if (band < 0) break;
     SAT_PADD(sm, kPfLbChunks, 1);
     const int32_t chunk = sm.tot_chunk[t];
+    // Chunk q is led by CTA q % CL; its gather slot and that slot's phase.
+    const uint32_t lead = q % CL;
+    const uint32_t m = q / CL;
+    const int ls = m % kNLead<P, CL>;
+    const uint32_t lph = (m / kNLead<P, CL>) & 1;
     // Arm the V_up receive before our aggregate can reach the leader.
     if (lane == 0) mbar_arrive_expect_tx(&sm.vin_full[t], kVecBytes);
-    if (rank == 0 && lane == 0) mbar_arrive_expect_tx(&sm.lead_full[t], CL * kVecBytes);
+    if (rank == lead && lane == 0) mbar_arrive_expect_tx(&sm.lead_full[ls], CL * kVecBytes);
     __syncwarp();
-    // This band's aggregate (sum of the warps' column totals) -> leader.
+    // This band's aggregate (sum of the warps' column totals) -> the chunk's leader.
     {
-      const uint32_t rbar = mapa(&sm.lead_full[t], 0);
+      const uint32_t rbar = mapa(&sm.lead_full[ls], lead);
 #pragma unroll
       for (int g = 0; g < C::G; ++g) {
         TB agg[C::E];
@@ -908,12 +921,11 @@ __device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p,
 #pragma unroll
           for (int e = 0; e < C::E; ++e) agg[e] += tt[e];
         }
-        st_async16(mapa(&sm.lead_in[t][rank][col_of<P>(g, lane)], 0), pack16<TB, C::E>(agg), rbar);
+        st_async16(mapa(&sm.lead_in[ls][rank][col_of<P>(g, lane)], lead), pack16<TB, C::E>(agg),
+                   rbar);
       }
     }
-    if (rank == 0) {
-      leader_chunk<P, CL>(sm, p, lbw, land_ph, t, q, band, sm.tot_img[t], sm.tot_k[t], chunk, lane);
-    }
+    if (rank == lead) leader_chunk<P, CL>(sm, p, lbw, land_ph, t, ls, lph, band - rank, chunk, lane);
     SAT_PT(t4);
     mbar_wait_cluster(&sm.vin_full[t], (q / NT) & 1);
     SAT_PT(t5);
@@ -1228,9 +1240,9 @@ __global__ void __launch_bounds__(kThreads, 2)
     for (int t = 0; t < kNTot<P>; ++t) {
       mbar_init(&sm.tot_full[t], kNCW);
       mbar_init(&sm.carry_full[t], 1);
-      mbar_init(&sm.lead_full[t], 1);
       mbar_init(&sm.vin_full[t], 1);
     }
+    for (int i = 0; i < kNLead<P, CL>; ++i) mbar_init(&sm.lead_full[i], 1);
     for (int i = 0; i < kNLB; ++i) mbar_init(&sm.land_full[i], 1);
     mbar_init(&sm.tk_full, 1);
     mbar_init(&sm.tk_empty, CL > 1 ? CL - 1 : 1);
