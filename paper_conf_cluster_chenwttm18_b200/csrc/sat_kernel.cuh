@@ -1055,14 +1055,27 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
                          off[g]);
     const int64_t k = sm.meta[warp][t][2];
     const int32_t chunk = sm.meta[warp][t][3];
-    char* obase = p.out + (int64_t)img * p.out_img_stride;
+    const int64_t y0 = k * C::TH + warp * RW;
     const int64_t x0 = (int64_t)chunk * C::TW;
+    char* orow = p.out + (int64_t)img * p.out_img_stride + y0 * p.out_pitch;
     tmem_wait_ld();
+    if (kVecOut && y0 + RW <= p.H && x0 + C::TW <= p.W) {
+      // interior tile rows: no edge predicates, row pointers by increment
 #pragma unroll
-    for (int i = 0; i < RW; ++i) {
-      const int64_t y = k * C::TH + warp * RW + i;
-      if (y < p.H) {
-        TB* orow = reinterpret_cast<TB*>(obase + y * p.out_pitch);
+      for (int i = 0; i < RW; ++i, orow += p.out_pitch) {
+#pragma unroll
+        for (int g = 0; g < C::G; ++g) {
+          TB v[C::E];
+#pragma unroll
+          for (int e = 0; e < C::E; ++e)
+            v[e] = off[g][e] + get_words<TB>(w, (i * C::G + g) * C::E + e);
+          st_cs_v4(reinterpret_cast<TB*>(orow) + x0 + col_of<P>(g, lane), pack16<TB, C::E>(v));
+        }
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < RW; ++i, orow += p.out_pitch) {
+        if (y0 + i >= p.H) break;
 #pragma unroll
         for (int g = 0; g < C::G; ++g) {
           TB v[C::E];
@@ -1070,12 +1083,13 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
           for (int e = 0; e < C::E; ++e)
             v[e] = off[g][e] + get_words<TB>(w, (i * C::G + g) * C::E + e);
           const int64_t x = x0 + col_of<P>(g, lane);
+          TB* o = reinterpret_cast<TB*>(orow);
           if (kVecOut && x + C::E <= p.W) {
-            st_cs_v4(orow + x, pack16<TB, C::E>(v));
+            st_cs_v4(o + x, pack16<TB, C::E>(v));
           } else {
 #pragma unroll
             for (int e = 0; e < C::E; ++e)
-              if (x + e < p.W) orow[x + e] = v[e];
+              if (x + e < p.W) o[x + e] = v[e];
           }
         }
       }

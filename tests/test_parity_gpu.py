@@ -334,3 +334,47 @@ def test_full_size_batch_1024_frames_sampled():
     for n in (0, 1, 511, 1023):
         ref = oracle.sat_gen_rows(0, H, W, list(range(H)), seed=1002, img=n)
         check(y[n].cpu().numpy(), ref, np.uint8, f"frame {n}")
+
+
+# ---------------------------------------------------------------------------
+# Launch-configuration variants: cluster sizes (bands per thread-block
+# cluster) and the generic (non-TMA) load path, selected per launch.
+
+@pytest.mark.parametrize("cluster", ["1", "4", "8"])
+@pytest.mark.parametrize("np_dtype", [np.uint8, np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(1, 1), (33, 257), (999, 1001), (1080, 1920), (4099, 4097)])
+def test_parity_cluster_sizes(monkeypatch, cluster, np_dtype, shape):
+    torch = _torch()
+    sat = _sat()
+    monkeypatch.setenv("SAT_CLUSTER", cluster)
+    H, W = shape
+    x = gen(np_dtype, H, W, seed=2001 + H)
+    y = sat.sat(x)
+    torch.cuda.synchronize()
+    check(y.cpu().numpy(), oracle.sat(x.cpu().numpy()), np_dtype, f"CL={cluster} {shape}")
+
+
+@pytest.mark.parametrize("cluster", ["1", "4", "8"])
+def test_batched_partial_clusters(monkeypatch, cluster):
+    """34 bands per 1080-row frame: clusters straddle frames (segmented scan)."""
+    torch = _torch()
+    sat = _sat()
+    monkeypatch.setenv("SAT_CLUSTER", cluster)
+    N, H, W = 7, 1080, 700
+    x = torch.empty((N, H, W), dtype=torch.uint8, device="cuda")
+    satgen.fill_device(x, seed=31)
+    y = sat.sat(x).cpu().numpy()
+    xn = x.cpu().numpy()
+    for n in range(N):
+        check(y[n], oracle.sat(xn[n]), np.uint8, f"CL={cluster} frame {n}")
+
+
+@pytest.mark.parametrize("np_dtype", [np.uint8, np.float32, np.float64])
+def test_generic_load_path_forced(monkeypatch, np_dtype):
+    torch = _torch()
+    sat = _sat()
+    monkeypatch.setenv("SAT_FORCE_GENERIC", "1")
+    x = gen(np_dtype, 777, 1333, seed=41)
+    y = sat.sat(x)
+    torch.cuda.synchronize()
+    check(y.cpu().numpy(), oracle.sat(x.cpu().numpy()), np_dtype, "generic")
