@@ -905,50 +905,31 @@ __device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p,
     // Arm the V_up receive before our aggregate can reach the leader.
     if (lane == 0) mbar_arrive_expect_tx(&sm.vin_full[t], kVecBytes);
     if (rank == lead && lane == 0) mbar_arrive_expect_tx(&sm.lead_full[ls], CL * kVecBytes);
-    __syncwarp();
-    // This band's aggregate (sum of the warps' column totals) -> the chunk's leader.
-    {
-      const uint32_t rbar = mapa(&sm.lead_full[ls], lead);
-#pragma unroll
-      for (int g = 0; g < C::G; ++g) {
-        TB agg[C::E];
-#pragma unroll
-        for (int e = 0; e < C::E; ++e) agg[e] = TB(0);
-#pragma unroll
-        for (int w = 0; w < kNCW; ++w) {
-          TB tt[C::E];
-          unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]), tt);
-#pragma unroll
-          for (int e = 0; e < C::E; ++e) agg[e] += tt[e];
-        }
-        st_async16(mapa(&sm.lead_in[ls][rank][col_of<P>(g, lane)], lead), pack16<TB, C::E>(agg),
-                   rbar);
-      }
-    }
-    if (rank == lead) leader_chunk<P, CL>(sm, p, lbw, land_ph, t, ls, lph, band - rank, chunk, lane);
-    SAT_PT(t4);
-    mbar_wait_cluster(&sm.vin_full[t], (q / NT) & 1);
-    SAT_PT(t5);
-    SAT_PADD(sm, kPfLbWaitV, t5 - t4);
-    TB V[C::G][C::E];
-#pragma unroll
-    for (int g = 0; g < C::G; ++g)
-      unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.vin[t][col_of<P>(g, lane)]), V[g]);
-    // Fix-up offsets, in place: tot[w] <- V + sum_{w' < w} tot[w'] (Fig. 3c step #2).
+    TB agg[C::G][C::E];
 #pragma unroll
     for (int g = 0; g < C::G; ++g) {
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) agg[g][e] = TB(0);
 #pragma unroll
       for (int w = 0; w < kNCW; ++w) {
         uint4* cell = reinterpret_cast<uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]);
         TB tt[C::E];
         unpack16<TB, C::E>(*cell, tt);
-        *cell = pack16<TB, C::E>(V[g]);
+        *cell = pack16<TB, C::E>(agg[g]);
 #pragma unroll
-        for (int e = 0; e < C::E; ++e) V[g][e] += tt[e];
+        for (int e = 0; e < C::E; ++e) agg[g][e] += tt[e];
       }
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&sm.carry_full[t]);
+    {
+      const uint32_t rbar = mapa(&sm.lead_full[ls], lead);
+#pragma unroll
+      for (int g = 0; g < C::G; ++g)
+        st_async16(mapa(&sm.lead_in[ls][rank][col_of<P>(g, lane)], lead), pack16<TB, C::E>(agg[g]),
+                   rbar);
+    }
+    if (rank == lead) leader_chunk<P, CL>(sm, p, lbw, land_ph, t, ls, lph, band - rank, chunk, lane);
   }
 }
 
@@ -1042,6 +1023,7 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   const int t = q % kNTot<P>;
   SAT_PT(t0);
   mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
+  mbar_wait_cluster(&sm.vin_full[t], (q / kNTot<P>) & 1);
   SAT_PT(t1);
   if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
   const int32_t img = sm.meta[warp][t][1];
@@ -1050,9 +1032,14 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
     tmem_ld(tmem_addr(sm, t, warp), w);
     TB off[C::G][C::E];
 #pragma unroll
-    for (int g = 0; g < C::G; ++g)
+    for (int g = 0; g < C::G; ++g) {
+      TB v[C::E];
       unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]),
                          off[g]);
+      unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.vin[t][col_of<P>(g, lane)]), v);
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) off[g][e] += v[e];
+    }
     const int64_t k = sm.meta[warp][t][2];
     const int32_t chunk = sm.meta[warp][t][3];
     const int64_t y0 = k * C::TH + warp * RW;
