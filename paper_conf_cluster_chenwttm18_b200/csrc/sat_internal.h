@@ -17,7 +17,7 @@ struct sat_plan_st {
   int64_t max_h = 0, max_w = 0, max_batch = 0;
   int num_sms = 0;
   int active_clusters[3][3][4] = {};  // [pair][cluster 1/4/8][mode: bit0 TMA, bit1 vec out]
-  int cluster = 4;                    // CTAs (bands) per cluster: 1, 4 or 8
+  int cluster = 0;                    // forced CTAs (bands) per cluster (0: by shape)
   int64_t max_tiles = 0;       // capacity of the look-back workspace in tiles
   void* ws = nullptr;
   size_t ws_bytes = 0;
