@@ -344,6 +344,25 @@ __device__ __forceinline__ void st_async16(uint32_t raddr, uint4 v, uint32_t rba
       : "memory");
 }
 
+// Expect `bytes` of tx on a local mbarrier without arriving.
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+
+// 16-byte hand-off into CTA `dst` of the cluster.  Remote: st.async with tx on
+// its mbarrier.  Self (st.async needs a remote CTA -- a cluster of 1 has
+// none): plain shared store; the caller then arrives (release) on the barrier,
+// which was armed for the remote bytes only.
+__device__ __forceinline__ void send16(void* local_dst, uint64_t* local_bar, uint32_t dst,
+                                       uint32_t self, uint4 v) {
+  if (dst == self)
+    *reinterpret_cast<uint4*>(local_dst) = v;
+  else
+    st_async16(mapa(local_dst, dst), v, mapa(local_bar, dst));
+}
+
 __device__ __forceinline__ void st_async8(uint32_t raddr, uint64_t v, uint32_t rbar) {
   asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b64 [%0], %1, [%2];" ::"r"(raddr),
                "l"(v), "r"(rbar)
@@ -635,11 +654,28 @@ __device__ __forceinline__ uint64_t* payload_row(const KParams& p, int64_t T, in
 // One vector per (cluster ticket, chunk): written first as the aggregate, then
 // overwritten in place by the inclusive prefix.  A reader classifies a vector
 // by its words' tags (all AGG, all INCL, or not ready / mixed -> re-read).
+// Debug builds (-DSAT_DEBUG_DELAY) sleep a pseudo-random 0..~4 us before every
+// carry publication, look-back round and DSMEM hand-off, so tests exercise
+// late predecessors, mixed aggregate/inclusive windows and retries.
+#ifdef SAT_DEBUG_DELAY
+__device__ __forceinline__ void debug_delay(uint32_t salt) {
+  uint32_t x = (uint32_t)clock64() ^ (salt * 0x9E3779B9u) ^ (blockIdx.x * 0x85EBCA6Bu);
+  x ^= x >> 16;
+  x *= 0x7FEB352Du;
+  x ^= x >> 15;
+  if ((x & 3u) == 0) __nanosleep((x >> 4) & 4095u);
+}
+#define SAT_DELAY(salt) debug_delay(salt)
+#else
+#define SAT_DELAY(salt)
+#endif
+
 template <int P>
 __device__ __forceinline__ void publish(const KParams& p, int64_t T, int32_t chunk, uint32_t st,
                                         const typename Cfg<P>::TB (&v)[Cfg<P>::G][Cfg<P>::E],
                                         int lane) {
   using C = Cfg<P>;
+  SAT_DELAY(st + 17u * chunk);
   uint64_t* row = payload_row<P>(p, T, chunk);
 #pragma unroll
   for (int g = 0; g < C::G; ++g) {
@@ -689,6 +725,7 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
     int kk = nb;  // index of the inclusive vector in this round (nb: none)
     for (;;) {
       __syncwarp();  // every lane is done reading the previous round's landing zone
+      SAT_DELAY(31u + (uint32_t)j);
       SAT_PT(i0);
       // lane b fetches vector b (parallel issue); lane 0 arms the barrier.  The
       // previous round's generic reads of the landing zone were consumed before
@@ -836,6 +873,7 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
   }
   // Pass 2: V_up of every band of the cluster (padding CTAs get zeros).
   {
+    const uint32_t self = CL > 1 ? cluster_rank() : 0u;
     TB run[C::G][C::E];
 #pragma unroll
     for (int g = 0; g < C::G; ++g)
@@ -850,7 +888,6 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
 #pragma unroll
           for (int e = 0; e < C::E; ++e) run[g][e] = carry0[g][e];
       }
-      const uint32_t rbar = mapa(&sm.vin_full[t], r);
 #pragma unroll
       for (int g = 0; g < C::G; ++g) {
         TB v[C::E], a[C::E];
@@ -863,7 +900,11 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
           v[e] = valid ? run[g][e] : TB(0);
           if (valid) run[g][e] += a[e];
         }
-        st_async16(mapa(&sm.vin[t][col_of<P>(g, lane)], r), pack16<TB, C::E>(v), rbar);
+        send16(&sm.vin[t][col_of<P>(g, lane)], &sm.vin_full[t], (uint32_t)r, self, pack16<TB, C::E>(v));
+      }
+      if ((uint32_t)r == self) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.vin_full[t]);
       }
       if (++k == bpi) k = 0;
     }
@@ -902,9 +943,17 @@ __device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p,
     const uint32_t m = q / CL;
     const int ls = m % kNLead<P, CL>;
     const uint32_t lph = (m / kNLead<P, CL>) & 1;
-    // Arm the V_up receive before our aggregate can reach the leader.
-    if (lane == 0) mbar_arrive_expect_tx(&sm.vin_full[t], kVecBytes);
-    if (rank == lead && lane == 0) mbar_arrive_expect_tx(&sm.lead_full[ls], CL * kVecBytes);
+    SAT_DELAY(7u * q + rank);
+    // Arm the V_up receive before our aggregate can reach the leader.  The
+    // leader's own hand-offs are shared stores + arrive (see send16), so it
+    // arms only the bytes of its CL-1 peers.
+    if (lane == 0) {
+      if (rank != lead) {
+        mbar_arrive_expect_tx(&sm.vin_full[t], kVecBytes);
+      } else if (CL > 1) {
+        mbar_expect_tx(&sm.lead_full[ls], (CL - 1) * kVecBytes);
+      }
+    }
     TB agg[C::G][C::E];
 #pragma unroll
     for (int g = 0; g < C::G; ++g) {
@@ -922,12 +971,13 @@ __device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p,
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&sm.carry_full[t]);
-    {
-      const uint32_t rbar = mapa(&sm.lead_full[ls], lead);
 #pragma unroll
-      for (int g = 0; g < C::G; ++g)
-        st_async16(mapa(&sm.lead_in[ls][rank][col_of<P>(g, lane)], lead), pack16<TB, C::E>(agg[g]),
-                   rbar);
+    for (int g = 0; g < C::G; ++g)
+      send16(&sm.lead_in[ls][rank][col_of<P>(g, lane)], &sm.lead_full[ls], lead, rank,
+             pack16<TB, C::E>(agg[g]));
+    if (lead == rank) {  // own contribution went by shared stores
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sm.lead_full[ls]);
     }
     if (rank == lead) leader_chunk<P, CL>(sm, p, lbw, land_ph, t, ls, lph, band - rank, chunk, lane);
   }
