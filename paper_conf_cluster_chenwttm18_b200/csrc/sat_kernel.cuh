@@ -82,7 +82,10 @@ struct Cfg<P8U32S> {
   static constexpr int G = 2;   // groups per lane: cols {4l..4l+3} and {128+4l..}
   static constexpr int TW = 32 * E * G;  // 256
   static constexpr int TH = 32;
-  static constexpr int LOOK = 3;         // pass B runs LOOK chunks behind pass A
+#ifndef SAT_LOOK8
+#define SAT_LOOK8 3
+#endif
+  static constexpr int LOOK = SAT_LOOK8;  // pass B runs LOOK chunks behind pass A
   static constexpr int NSTAGE = 4;       // TMA prefetch depth (stages free after pass A)
 };
 template <>
@@ -93,7 +96,10 @@ struct Cfg<P32F32F> {
   static constexpr int G = 1;
   static constexpr int TW = 128;
   static constexpr int TH = 32;
-  static constexpr int LOOK = 4;
+#ifndef SAT_LOOK32
+#define SAT_LOOK32 7
+#endif
+  static constexpr int LOOK = SAT_LOOK32;
   static constexpr int NSTAGE = 3;
 };
 template <>
@@ -104,7 +110,10 @@ struct Cfg<P64F64F> {
   static constexpr int G = 1;
   static constexpr int TW = 64;
   static constexpr int TH = 32;
-  static constexpr int LOOK = 4;
+#ifndef SAT_LOOK64
+#define SAT_LOOK64 4
+#endif
+  static constexpr int LOOK = SAT_LOOK64;
   static constexpr int NSTAGE = 3;
 };
 
@@ -166,6 +175,17 @@ __device__ __forceinline__ uint64_t gtime() {
 #else
 #define SAT_PT(v)
 #define SAT_PADD(sm_, slot_, val_)
+#endif
+// Optional timeline (debug builds with -DSAT_TIMELINE): globaltimer at every
+// pass B of the first band each CTA processes, plus that band's index.
+#ifdef SAT_TIMELINE
+constexpr int kTlChunks = 256;
+__device__ unsigned long long g_sat_tl[1024][2 + kTlChunks];
+__device__ __forceinline__ uint64_t tl_now() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 #endif
 enum ProfSlot {
   kPfComputeWaitFull = 0,   // warp 0: waiting for TMA data
@@ -864,7 +884,15 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
     }
   }
   TB Vcl[C::G][C::E];
+#ifdef SAT_DEBUG_NO_LOOKBACK  // timing experiments only: wrong results, no cross-cluster wait
+#pragma unroll
+  for (int g = 0; g < C::G; ++g)
+#pragma unroll
+    for (int e = 0; e < C::E; ++e) Vcl[g][e] = TB(0);
+  if (false) {
+#else
   if (!head_self) {
+#endif
     SAT_PT(t2);
     const int64_t first = ((int64_t)n0 * bpi) / CL;
     lookback<P>(sm, sm.land[lbw], &sm.land_full[lbw], land_ph, p, T, first, chunk, Vcl, lane);
@@ -1134,6 +1162,14 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   }
   SAT_PT(t2);
   if (warp == 0) SAT_PADD(sm, kPfComputeFixup, t2 - t1);
+#ifdef SAT_TIMELINE
+  if (warp == 0 && lane == 0 && blockIdx.x < 1024 && img >= 0 && q < kTlChunks &&
+      q < (uint32_t)p.nchunks) {
+    if (q == 0) g_sat_tl[blockIdx.x][1] = (unsigned long long)sm.meta[0][t][2] +
+                                          ((unsigned long long)img << 32);
+    g_sat_tl[blockIdx.x][2 + q] = tl_now();
+  }
+#endif
 }
 
 template <int P, int CL, bool kVecOut>
@@ -1320,6 +1356,9 @@ __global__ void __launch_bounds__(kThreads, 2)
     __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 
+#ifdef SAT_TIMELINE
+  if (threadIdx.x == 0 && blockIdx.x < 1024) g_sat_tl[blockIdx.x][0] = tl_now();
+#endif
   if (warp == kProducerWarp) {
     producer_warp<P, CL, kTMA>(sm, p, &map, rank, lane);
   } else if (warp >= kFirstLbWarp) {

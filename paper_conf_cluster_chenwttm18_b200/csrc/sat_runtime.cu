@@ -171,6 +171,28 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
+#ifdef SAT_TIMELINE
+  {
+    static unsigned long long tl[1024][2 + kTlChunks];
+    cudaStreamSynchronize(stream);
+    cudaMemcpyFromSymbol(tl, g_sat_tl, sizeof(tl));
+    static unsigned long long zero[1024][2 + kTlChunks];
+    cudaMemcpyToSymbol(g_sat_tl, zero, sizeof(zero));
+    const char* path = getenv("SAT_TIMELINE_OUT");
+    FILE* f = path ? fopen(path, "a") : nullptr;
+    if (f) {
+      fprintf(f, "launch pair=%d h=%lld w=%lld batch=%lld CL=%d grid=%lld nchunks=%d\n", P,
+              (long long)h, (long long)w, (long long)batch, CL, (long long)grid, kp.nchunks);
+      const int nc = std::min<int>(kp.nchunks, kTlChunks);
+      for (int64_t b = 0; b < grid && b < 1024; ++b) {
+        fprintf(f, "cta %lld %llu %llu", (long long)b, tl[b][0], tl[b][1]);
+        for (int c = 0; c < nc; ++c) fprintf(f, " %llu", tl[b][2 + c]);
+        fprintf(f, "\n");
+      }
+      fclose(f);
+    }
+  }
+#endif
 #ifdef SAT_PROFILE
   {
     unsigned long long prof[16];
