@@ -346,6 +346,10 @@ def run_ours(args, workload, rank, world, local_rank):
                "steps": e2e_steps, "path": "sat_compute_host (pinned host in/out, banded H2D/SAT/D2H overlap)"}
         del xh, oh
 
+    banded = None
+    if world > 1 or args.banded:
+        banded = run_banded(args, rank, world, local_rank)
+
     if rank != 0:
         return
     line = {
@@ -366,6 +370,8 @@ def run_ours(args, workload, rank, world, local_rank):
         "clocks": sampler.summary() | {"remeasured": remeasured},
         "e2e": e2e,
     }
+    if banded is not None:
+        line["banded"] = banded
     if world == 1 and not args.no_sweep:
         sweep = []
         for (p_, h_, w_, n_) in [(0, 1024, 1024, 1), (0, 2048, 2048, 1), (0, 4096, 4096, 1),
@@ -386,6 +392,70 @@ def run_ours(args, workload, rank, world, local_rank):
     print(json.dumps(line), flush=True)
 
 
+def run_banded(args, rank, world, local_rank, H=65536, W=65536, pair=1, seed=1004):
+    """BASELINE configs[3]: ONE 65536 x 65536 32f image row-banded across the
+    ranks (sat_compute_dist: band column sums -> ncclAllGather of the W-vectors
+    -> carry row -> band SAT with the carry fused).  Timed like the headline
+    (barrier + events on the launching stream, max over ranks); value = the
+    whole image's pixels / step time."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cluster_chenwttm18_b200 as sat
+    import satgen
+
+    dev = torch.device("cuda", local_rank)
+    own_pg = False
+    if not dist.is_initialized():  # N = 1: a one-rank group to bootstrap the NCCL comm
+        import socket
+        so = socket.socket()
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+        so.close()
+        dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
+        own_pg = True
+    r0, r1 = sat.band_partition(H, world, rank)
+    dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64}[pair]
+    band = torch.empty((r1 - r0, W), dtype=dt, device=dev)
+    satgen.fill_device(band, seed=seed, y0=r0)
+    out = torch.empty((r1 - r0, W), dtype=sat.out_dtype(pair), device=dev)
+    plan = sat.Plan(pair, max(r1 - r0, 1), W, 1, dev)
+    comm = sat.SatComm(device=dev)
+    s = torch.cuda.current_stream(dev)
+    steps = max(3, min(args.steps, 10))
+    for _ in range(max(3, args.warmup)):
+        sat.sat_dist(band, comm, out=out, plan=plan)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(s)
+    for _ in range(steps):
+        sat.sat_dist(band, comm, out=out, plan=plan)
+    b.record(s)
+    torch.cuda.synchronize()
+    ms = a.elapsed_time(b) / steps
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        dist.barrier()
+    comm.close()
+    if own_pg:
+        dist.destroy_process_group()
+    del band, out
+    torch.cuda.empty_cache()
+    px = H * W
+    # per rank: the band is read twice (column sums, then the SAT) and written once
+    per_rank_bytes = (r1 - r0) * W * (2 * IN_B[pair] + OUT_B[pair])
+    return {"workload": "huge-65536sq-32f32f row-banded", "n_gpus": world, "steps": steps,
+            "ms_per_step": ms, "value": px / (ms * 1e-3) / 1e9, "unit": "Gpx/s",
+            "scaling": "strong", "parallelism": f"row bands x{world} (ncclAllGather carry)",
+            "rank0_band_rows": r1 - r0, "hbm_bytes_per_rank": per_rank_bytes,
+            "rank_gbs": per_rank_bytes / (ms * 1e-3) / 1e9}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -394,6 +464,8 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD, choices=sorted(WORKLOADS))
     ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--banded", action="store_true",
+                    help="also time the row-banded 65536^2 32f path (always on for N > 1)")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))

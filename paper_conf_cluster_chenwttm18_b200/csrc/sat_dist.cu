@@ -352,6 +352,11 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
   }
   DeviceGuard g(plan->device);
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (comm->nranks == 1) {  // one band = the whole image: no carry to exchange
+    if (band_h == 0) return SAT_OK;
+    return launch(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
+                  band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1, nullptr, s);
+  }
   DistBufs& b = comm->bufs;
   sat_status st = ensure_bufs(b, w, comm->nranks);
   if (st != SAT_OK) return st;

@@ -59,14 +59,10 @@ namespace sat {
 
 enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2 };
 
-constexpr int kNCW = 8;                          // compute warps
 #ifndef SAT_NLB
 #define SAT_NLB 3
 #endif
 constexpr int kNLB = SAT_NLB;                    // look-back warps
-constexpr int kProducerWarp = kNCW;
-constexpr int kFirstLbWarp = kNCW + 1;
-constexpr int kThreads = (kNCW + 1 + kNLB) * 32;
 constexpr uint32_t kFull = 0xffffffffu;
 
 // Carry word tag (high 32 bits): (epoch << 2) | st,  st: 1 aggregate, 2 inclusive.
@@ -86,7 +82,11 @@ struct Cfg<P8U32S> {
 #define SAT_LOOK8 3
 #endif
   static constexpr int LOOK = SAT_LOOK8;  // pass B runs LOOK chunks behind pass A
-  static constexpr int NSTAGE = 4;       // TMA prefetch depth (stages free after pass A)
+#ifndef SAT_NCW8
+#define SAT_NCW8 8
+#endif
+  static constexpr int NCW = SAT_NCW8;   // compute warps (TH / NCW rows each)
+  static constexpr int NSTAGE = NCW > 8 ? 3 : 4;  // TMA prefetch depth (stages free after pass A)
 };
 template <>
 struct Cfg<P32F32F> {
@@ -100,6 +100,7 @@ struct Cfg<P32F32F> {
 #define SAT_LOOK32 7
 #endif
   static constexpr int LOOK = SAT_LOOK32;
+  static constexpr int NCW = 8;
   static constexpr int NSTAGE = 3;
 };
 template <>
@@ -114,8 +115,19 @@ struct Cfg<P64F64F> {
 #define SAT_LOOK64 4
 #endif
   static constexpr int LOOK = SAT_LOOK64;
+  static constexpr int NCW = 8;
   static constexpr int NSTAGE = 3;
 };
+
+// Warp roles: NCW compute warps, then the producer, then kNLB look-back warps.
+template <int P>
+constexpr int kNCW = Cfg<P>::NCW;
+template <int P>
+constexpr int kProducerWarp = kNCW<P>;
+template <int P>
+constexpr int kFirstLbWarp = kNCW<P> + 1;
+template <int P>
+constexpr int kThreads = (kNCW<P> + 1 + kNLB) * 32;
 
 // Words of one carry payload vector: TW elements * (4 / E) 64-bit words per element.
 template <int P>
@@ -135,10 +147,10 @@ constexpr int kNTot = (Cfg<P>::LOOK + 1 > kNLB) ? Cfg<P>::LOOK + 1 : kNLB;  // >
 // per warp and chunk slot, RW rows x G x E values of 32-bit words (fp64: 2 words).
 template <int P>
 constexpr int kTmemColsPerWarp =
-    (Cfg<P>::TH / kNCW) * Cfg<P>::G * Cfg<P>::E * (int)(sizeof(typename Cfg<P>::TB) / 4);
+    (Cfg<P>::TH / kNCW<P>) * Cfg<P>::G * Cfg<P>::E * (int)(sizeof(typename Cfg<P>::TB) / 4);
 constexpr int kTmemCols = 256;  // per CTA (2 CTAs per SM share the SM's 512 columns)
 template <int P>
-constexpr int kTmemColsPerSlot = kTmemColsPerWarp<P> * (kNCW / 4);  // 2 warps per subpartition
+constexpr int kTmemColsPerSlot = kTmemColsPerWarp<P> * (kNCW<P> / 4);  // NCW/4 warps per subpartition
 static_assert(kTmemColsPerSlot<P8U32S> * kNTot<P8U32S> <= kTmemCols, "TMEM budget (8u)");
 static_assert(kTmemColsPerSlot<P32F32F> * kNTot<P32F32F> <= kTmemCols, "TMEM budget (32f)");
 static_assert(kTmemColsPerSlot<P64F64F> * kNTot<P64F64F> <= kTmemCols, "TMEM budget (64f)");
@@ -217,10 +229,10 @@ template <int P, int CL>
 struct __align__(128) Smem {
   using C = Cfg<P>;
   typename C::TA in[C::NSTAGE][C::TH][C::TW];   // TMA destination ring
-  alignas(128) typename C::TB tot[kNTot<P>][kNCW][C::TW];    // per-warp column totals -> fix-up offsets
+  alignas(128) typename C::TB tot[kNTot<P>][kNCW<P>][C::TW];    // per-warp column totals -> fix-up offsets
   alignas(128) typename C::TB lead_in[kNLead<P, CL>][CL][C::TW];  // chunk leader: the bands' aggregates
   alignas(128) typename C::TB vin[kNTot<P>][C::TW];          // V_up of this band (from the leader)
-  int32_t meta[kNCW][kNTot<P>][4];              // per warp: (band lo, img, k, chunk) of each slot
+  int32_t meta[kNCW<P>][kNTot<P>][4];              // per warp: (band lo, img, k, chunk) of each slot
   uint32_t tmem_base;                           // TMEM address from tcgen05.alloc
   alignas(128) uint64_t land[kNLB][kLandVecs<P>][kVecWords<P>];  // look-back payload landing (bulk copies)
   uint64_t full[C::NSTAGE];
@@ -988,7 +1000,7 @@ __device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p,
 #pragma unroll
       for (int e = 0; e < C::E; ++e) agg[g][e] = TB(0);
 #pragma unroll
-      for (int w = 0; w < kNCW; ++w) {
+      for (int w = 0; w < kNCW<P>; ++w) {
         uint4* cell = reinterpret_cast<uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]);
         TB tt[C::E];
         unpack16<TB, C::E>(*cell, tt);
@@ -1027,11 +1039,11 @@ __device__ __forceinline__ uint32_t tmem_addr(const Smem<P, CL>& sm, int t, int 
 // the end-of-work sentinel.
 template <int P, int CL>
 __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint32_t ph,
-                                       typename Cfg<P>::TB (&rowcarry)[Cfg<P>::TH / kNCW],
+                                       typename Cfg<P>::TB (&rowcarry)[Cfg<P>::TH / kNCW<P>],
                                        int warp, int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
-  constexpr int RW = C::TH / kNCW;
+  constexpr int RW = C::TH / kNCW<P>;
   constexpr int NW = kTmemColsPerWarp<P>;
   SAT_PT(t0);
   mbar_wait(&sm.full[s], ph);
@@ -1096,7 +1108,7 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
                                        int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
-  constexpr int RW = C::TH / kNCW;
+  constexpr int RW = C::TH / kNCW<P>;
   constexpr int NW = kTmemColsPerWarp<P>;
   const int t = q % kNTot<P>;
   SAT_PT(t0);
@@ -1177,7 +1189,7 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
                                              int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
-  constexpr int RW = C::TH / kNCW;
+  constexpr int RW = C::TH / kNCW<P>;
   TB rowcarry[RW];
 #pragma unroll
   for (int i = 0; i < RW; ++i) rowcarry[i] = TB(0);
@@ -1310,7 +1322,7 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
 // ---------------------------------------------------------------------------
 
 template <int P, int CL, bool kTMA, bool kVecOut>
-__global__ void __launch_bounds__(kThreads, 2)
+__global__ void __launch_bounds__(kThreads<P>, 2)
     sat_tile_kernel(const __grid_constant__ CUtensorMap map, const KParams p) {
   using C = Cfg<P>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -1322,10 +1334,10 @@ __global__ void __launch_bounds__(kThreads, 2)
   if (threadIdx.x == 0) {
     for (int s = 0; s < C::NSTAGE; ++s) {
       mbar_init(&sm.full[s], 1);
-      mbar_init(&sm.empty[s], kNCW);
+      mbar_init(&sm.empty[s], kNCW<P>);
     }
     for (int t = 0; t < kNTot<P>; ++t) {
-      mbar_init(&sm.tot_full[t], kNCW);
+      mbar_init(&sm.tot_full[t], kNCW<P>);
       mbar_init(&sm.carry_full[t], 1);
       mbar_init(&sm.vin_full[t], 1);
     }
@@ -1359,10 +1371,10 @@ __global__ void __launch_bounds__(kThreads, 2)
 #ifdef SAT_TIMELINE
   if (threadIdx.x == 0 && blockIdx.x < 1024) g_sat_tl[blockIdx.x][0] = tl_now();
 #endif
-  if (warp == kProducerWarp) {
+  if (warp == kProducerWarp<P>) {
     producer_warp<P, CL, kTMA>(sm, p, &map, rank, lane);
-  } else if (warp >= kFirstLbWarp) {
-    lookback_warp<P, CL>(sm, p, warp - kFirstLbWarp, rank, lane);
+  } else if (warp >= kFirstLbWarp<P>) {
+    lookback_warp<P, CL>(sm, p, warp - kFirstLbWarp<P>, rank, lane);
   } else {
     compute_warp<P, CL, kVecOut>(sm, p, warp, lane);
   }

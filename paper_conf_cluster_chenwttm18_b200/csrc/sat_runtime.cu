@@ -144,7 +144,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
 
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
-  cfg.blockDim = dim3(kThreads);
+  cfg.blockDim = dim3(kThreads<P>);
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
@@ -255,7 +255,7 @@ int getenv_int(const char* name, int dflt) {
 // block size, dynamic shared memory, cluster shape and register bound, so its
 // answer is the real residency, which is then capped by TMEM.
 template <int P, int CL>
-__global__ void __launch_bounds__(kThreads, 2) sat_occupancy_proxy(int* sink) {
+__global__ void __launch_bounds__(kThreads<P>, 2) sat_occupancy_proxy(int* sink) {
   extern __shared__ unsigned char s[];
   if (sink) sink[threadIdx.x] = s[threadIdx.x];
 }
@@ -274,7 +274,7 @@ static sat_status configure_cl(sat_plan_st* pl) {
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(CL * 64);
-    cfg.blockDim = dim3(kThreads);
+    cfg.blockDim = dim3(kThreads<P>);
     cfg.dynamicSmemBytes = smem;
     cudaLaunchAttribute attr;
     attr.id = cudaLaunchAttributeClusterDimension;

@@ -14,6 +14,8 @@ for line in open(sys.argv[1]):
 for key, (hdr, ctas) in launches.items():
     t0 = min(c[1] for c in ctas)
     print(hdr)
+    st = sorted((c[1] - t0) / 1e3 for c in ctas if c[1])
+    print("  CTA start (us): min %.1f p50 %.1f p90 %.1f max %.1f  (n=%d)" % (st[0], st[len(st)//2], st[int(len(st)*0.9)], st[-1], len(st)))
     rows = sorted(((c[2] & 0xffffffff) + (c[2] >> 32) * 100000, c) for c in ctas if c[3] and c[3][0])
     nc = len(rows[0][1][3])
     cols = sorted(set([0, 1, 2, 4, 8, 16, 32, 48, nc - 1]) & set(range(nc)))
