@@ -118,3 +118,52 @@ def sat_gen_rows(pair: int, H: int, W: int, rows, seed: int = 0, img: int = 0, m
     _check(lib().oracle_sat_gen_rows(pair, mode, seed, img, value, H, W, rows.ctypes.data,
                                      len(rows), out.ctypes.data), "oracle_sat_gen_rows")
     return out
+
+
+def sat_exclusive(A: np.ndarray, full: bool = True, nval=0) -> np.ndarray:
+    """Exclusive SAT, PAPER.md:63-68 (Eq. 2): J(y, x) = 0 where x = 0 or y = 0,
+    else sum_{j < y} sum_{i < x} I(j, i); plus NPP's offset nVal on every
+    element (nppi_statistics_functions.h, nppiIntegral: pDst(j,i) = nVal +
+    sum_{l<j} sum_{k<i} pSrc(l,k)).
+
+    full=True: the (H+1) x (W+1) layout of NPP / OpenCV,
+    whose last row/column hold the totals; full=False: Eq. 2 as printed, the
+    same H x W size as I (reading R7 of DESIGN.md).  Built from the inclusive
+    oracle: J(y+1, x+1) = S(y, x) (Eq. 1 vs Eq. 2).  8u: int64 sum + nVal,
+    reported mod 2^32 as int32 (reading R2); floats: fp64 (64f: the
+    double-double inclusive result, + nVal rounded once).
+    """
+    assert A.ndim == 2
+    pair = pair_of(A)
+    H, W = A.shape
+    S = sat(A) if A.size else np.empty((H, W), dtype=OUT_DTYPE[pair])
+    if pair == PAIR_8U32S:
+        J = np.zeros((H + 1, W + 1), dtype=np.int64)
+        J[1:, 1:] = S.astype(np.int64)
+        J = (J + int(nval)) & 0xFFFFFFFF
+        J = J.astype(np.uint32).view(np.int32)
+    else:
+        J = np.zeros((H + 1, W + 1), dtype=np.float64)
+        J[1:, 1:] = S
+        J = J + float(nval)
+    return J if full else np.ascontiguousarray(J[:H, :W])
+
+
+def sat_exclusive_brute(A: np.ndarray, full: bool = True, nval=0) -> np.ndarray:
+    """Eq. 2 evaluated literally (tiny inputs only): every element is the
+    direct sum over its rectangle {j < y, i < x}, exact (Python ints /
+    fractions of the fp values), + nVal."""
+    from fractions import Fraction
+    H, W = A.shape
+    Hn, Wn = (H + 1, W + 1) if full else (H, W)
+    pair = pair_of(A)
+    vals = [[int(v) if pair == PAIR_8U32S else Fraction(float(v)) for v in row] for row in A]
+    out = np.zeros((Hn, Wn), dtype=np.int32 if pair == PAIR_8U32S else np.float64)
+    for y in range(Hn):
+        for x in range(Wn):
+            s = sum((vals[j][i] for j in range(y) for i in range(x)), 0)
+            if pair == PAIR_8U32S:
+                out[y, x] = np.uint32((s + int(nval)) & 0xFFFFFFFF).view(np.int32)
+            else:
+                out[y, x] = float(s + Fraction(float(nval)))
+    return out
