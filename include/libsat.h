@@ -116,6 +116,27 @@ sat_status sat_compute_host(sat_plan plan, const void* in_host, void* out_host, 
                             int64_t w, int64_t in_pitch_bytes, int64_t out_pitch_bytes,
                             sat_pair pair, void* stream);
 
+/* Exclusive SAT (Eq. 2) with NPP's offset nVal
+ * (nppiIntegral: pDst(j,i) = nVal + sum_{l<j} sum_{k<i}
+ * pSrc(l,k)):
+ *   J(y, x) = nVal                                   if x == 0 or y == 0
+ *   J(y, x) = nVal + sum_{j<y} sum_{i<x} A(j, i)     otherwise.
+ * full = 1: the (h+1) x (w+1) layout of NPP / OpenCV (last row and column
+ *           hold the totals) -- a drop-in nppiIntegral_8u32s_C1R replacement
+ *           for 8u->32s (in-place forbidden: J is shifted by one row/column);
+ * full = 0: Eq. 2 as printed, an h x w output (the full layout cropped).
+ * `out` (device) has out_pitch_bytes >= (w + full) * sizeof(T_B); nval points
+ * to ONE host value of T_B (int32 / float / double), NULL means 0.  The first
+ * row is filled by a small kernel, every other element by the single-pass SAT
+ * kernel, which stores S(y, x) at (y + 1, x + 1) with 16-byte aligned vector
+ * stores when `out` and the pitch are 16-byte aligned.  Asynchronous on
+ * `stream`; validation as sat_compute, plus SAT_ERR_UNSUPPORTED on any
+ * overlap of input and output.  h == 0 or w == 0 fills the border (full) or
+ * is a no-op (Eq. 2). */
+sat_status sat_compute_exclusive(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                                 int64_t in_pitch_bytes, int64_t out_pitch_bytes, int full,
+                                 const void* nval, sat_pair pair, void* stream);
+
 /* ---------------------------------------------------------------------------
  * Multi-GPU (one process per GPU, NCCL over NVLink/NVSwitch).
  * NCCL is loaded at run time (dlopen "libnccl.so.2"; the copy torch already

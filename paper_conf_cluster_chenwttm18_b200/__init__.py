@@ -57,6 +57,7 @@ def lib():
                     "sat_compute_batched": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_band": ([vp, vp, vp, i64, i64, i64, i64, vp, i32, vp], i32),
                     "sat_compute_host": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
+                    "sat_compute_exclusive": ([vp, vp, vp, i64, i64, i64, i64, i32, vp, i32, vp], i32),
                     "sat_comm_unique_id": ([vp], i32),
                     "sat_comm_create": ([ctypes.POINTER(vp), vp, i32, i32, i32], i32),
                     "sat_comm_destroy": ([vp], i32),
@@ -216,6 +217,34 @@ def sat(x, out=None, plan: Plan | None = None, stream=None):
         p.compute_batched_ptr(x.data_ptr(), out.data_ptr(), H, W, ip, op, iis, ois, N, stream)
     else:
         p.compute_ptr(x.data_ptr(), out.data_ptr(), H, W, ip, op, stream)
+    return out
+
+
+def sat_exclusive(x, full: bool = True, nval=0, out=None, plan: Plan | None = None, stream=None):
+    """Exclusive SAT (Eq. 2) of a CUDA tensor [H, W] plus nVal on every
+    element: full=True gives NPP's / OpenCV's (H+1) x (W+1) layout, full=False
+    Eq. 2's H x W.  sat_compute_exclusive does all the work."""
+    torch = _torch()
+    if not x.is_cuda or x.dim() != 2:
+        raise ValueError("sat_exclusive() needs a 2-D CUDA tensor")
+    pair = pair_of_dtype(x.dtype)
+    H, W = x.shape
+    shape = (H + 1, W + 1) if full else (H, W)
+    if out is None:
+        out = torch.empty(shape, dtype=out_dtype(pair), device=x.device)
+    elif out.dtype != out_dtype(pair) or tuple(out.shape) != shape or out.device != x.device:
+        raise ValueError("out has the wrong dtype/shape/device")
+    if out.numel() == 0:
+        return out
+    ctype = {0: ctypes.c_int32, 1: ctypes.c_float, 2: ctypes.c_double}[pair]
+    nv = ctype(nval)
+    ip = _row_layout(x)[0] if H > 0 and W > 0 else max(W, 1) * x.element_size()
+    op = _row_layout(out)[0]
+    p = plan if plan is not None else _plan_for(x.device, pair, max(H, 1), max(W, 1), 1)
+    _check(lib().sat_compute_exclusive(p.handle, x.data_ptr() if x.numel() else None,
+                                       out.data_ptr(), H, W, ip, op, 1 if full else 0,
+                                       ctypes.byref(nv), pair, _stream_ptr(stream, x.device)),
+           "sat_compute_exclusive")
     return out
 
 

@@ -44,9 +44,15 @@ int tile_h(sat_pair p);
 sat_status validate(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                     int64_t op, int64_t iis, int64_t ois, int64_t batch, sat_pair pair,
                     bool* empty);
+// Exclusive-layout output (sat_compute_exclusive): `out` points at output
+// row 1; S(y, x) lands in column x + 1 (< out_cols); every value gets nVal.
+struct ExSpec {
+  int64_t out_cols;
+  uint64_t nval_bits;
+};
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
-                  cudaStream_t stream);
+                  cudaStream_t stream, const ExSpec* ex = nullptr);
 void host_path_release(sat_plan_st* pl);
 
 struct DeviceGuard {

@@ -170,6 +170,11 @@ struct KParams {
   unsigned long long* counter;           // ticket counter (workspace)
   void* payload;                         // [tickets][nchunks][kVecWords] status-tagged carries
   const void* carry_in;                  // optional S(r0-1, .) row (W elems of TB) for image starts
+  // Exclusive layout (kernels instantiated with kEx): S(y, x) is stored at
+  // output row y (out already points at row 1 of the exclusive array) and
+  // column x + 1; column 0 holds nval; columns >= out_cols are not written.
+  int64_t out_cols;
+  uint64_t nval_bits;                    // nVal, a TB value's bits (added to every element)
 };
 
 // Optional phase profiling (debug builds with -DSAT_PROFILE): per-CTA shared
@@ -1103,9 +1108,55 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint3
 
 // Pass B of chunk q: wait for the fix-up offsets, load S' back from TMEM,
 // add, store (a8).
-template <int P, int CL, bool kVecOut>
+template <typename TB>
+__device__ __forceinline__ TB from_bits(uint64_t b) {
+  TB v;
+  memcpy(&v, &b, sizeof(TB));
+  return v;
+}
+
+// Exclusive-layout store of one tile row (Eq. 2; NPP layout):
+// S(y, x) goes to output column o = x + 1.  The 16-B aligned output vector of
+// lane l / group g starts at o0 = x0 + col_of(g, l) and holds S(x = o0 - 1 ..
+// o0 + E - 2): the previous lane's last element, then this lane's first E - 1.
+// Lane 0 takes its first element from group g - 1 (lane 31) or, for g = 0, from
+// the previous chunk (`prevlast`, nVal at chunk 0 = output column 0).
+template <int P, bool kVecOut>
+__device__ __forceinline__ void store_row_exclusive(
+    const KParams& p, char* orow, int64_t x0, bool last_chunk,
+    const typename Cfg<P>::TB (&v)[Cfg<P>::G][Cfg<P>::E], typename Cfg<P>::TB& prevlast, int lane) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  TB sh[C::G][C::E];
+#pragma unroll
+  for (int g = 0; g < C::G; ++g) {
+    const TB up = __shfl_up_sync(kFull, v[g][C::E - 1], 1);
+    const TB l31 = g > 0 ? __shfl_sync(kFull, v[g > 0 ? g - 1 : 0][C::E - 1], 31) : prevlast;
+    sh[g][0] = lane == 0 ? l31 : up;
+#pragma unroll
+    for (int e = 1; e < C::E; ++e) sh[g][e] = v[g][e - 1];
+  }
+  const TB newlast = __shfl_sync(kFull, v[C::G - 1][C::E - 1], 31);
+  TB* o = reinterpret_cast<TB*>(orow);
+#pragma unroll
+  for (int g = 0; g < C::G; ++g) {
+    const int64_t o0 = x0 + col_of<P>(g, lane);
+    if (kVecOut && o0 + C::E <= p.out_cols) {
+      st_cs_v4(o + o0, pack16<TB, C::E>(sh[g]));
+    } else {
+#pragma unroll
+      for (int e = 0; e < C::E; ++e)
+        if (o0 + e < p.out_cols) o[o0 + e] = sh[g][e];
+    }
+  }
+  // W a multiple of TW: the last column (o = W) lies past this chunk's vectors.
+  if (last_chunk && lane == 31 && x0 + C::TW < p.out_cols) o[x0 + C::TW] = newlast;
+  prevlast = newlast;
+}
+
+template <int P, int CL, bool kVecOut, bool kEx>
 __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32_t q, int warp,
-                                       int lane) {
+                                       int lane, typename Cfg<P>::TB (&prevlast)[Cfg<P>::TH / kNCW<P>]) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr int RW = C::TH / kNCW<P>;
@@ -1129,6 +1180,10 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
       unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.vin[t][col_of<P>(g, lane)]), v);
 #pragma unroll
       for (int e = 0; e < C::E; ++e) off[g][e] += v[e];
+      if constexpr (kEx) {
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) off[g][e] += from_bits<TB>(p.nval_bits);
+      }
     }
     const int64_t k = sm.meta[warp][t][2];
     const int32_t chunk = sm.meta[warp][t][3];
@@ -1136,7 +1191,24 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
     const int64_t x0 = (int64_t)chunk * C::TW;
     char* orow = p.out + (int64_t)img * p.out_img_stride + y0 * p.out_pitch;
     tmem_wait_ld();
-    if (kVecOut && y0 + RW <= p.H && x0 + C::TW <= p.W) {
+    if constexpr (kEx) {
+      if (chunk == 0) {
+#pragma unroll
+        for (int i = 0; i < RW; ++i) prevlast[i] = from_bits<TB>(p.nval_bits);
+      }
+      const bool last_chunk = chunk == p.nchunks - 1;
+#pragma unroll
+      for (int i = 0; i < RW; ++i, orow += p.out_pitch) {
+        if (y0 + i >= p.H) break;  // warp-uniform
+        TB v[C::G][C::E];
+#pragma unroll
+        for (int g = 0; g < C::G; ++g)
+#pragma unroll
+          for (int e = 0; e < C::E; ++e)
+            v[g][e] = off[g][e] + get_words<TB>(w, (i * C::G + g) * C::E + e);
+        store_row_exclusive<P, kVecOut>(p, orow, x0, last_chunk, v, prevlast[i], lane);
+      }
+    } else if (kVecOut && y0 + RW <= p.H && x0 + C::TW <= p.W) {
       // interior tile rows: no edge predicates, row pointers by increment
 #pragma unroll
       for (int i = 0; i < RW; ++i, orow += p.out_pitch) {
@@ -1184,12 +1256,13 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
 #endif
 }
 
-template <int P, int CL, bool kVecOut>
+template <int P, int CL, bool kVecOut, bool kEx>
 __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, int warp,
                                              int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   constexpr int RW = C::TH / kNCW<P>;
+  TB prevlast[RW];  // exclusive layout: each row's last value of the previous chunk
   TB rowcarry[RW];
 #pragma unroll
   for (int i = 0; i < RW; ++i) rowcarry[i] = TB(0);
@@ -1203,7 +1276,7 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
         ended = true;
     }
     if (qb < qa && (ended || qa - qb > (uint32_t)C::LOOK)) {
-      pass_b<P, CL, kVecOut>(sm, p, qb, warp, lane);
+      pass_b<P, CL, kVecOut, kEx>(sm, p, qb, warp, lane, prevlast);
       ++qb;
     } else if (ended) {
       break;
@@ -1321,7 +1394,7 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
 
 // ---------------------------------------------------------------------------
 
-template <int P, int CL, bool kTMA, bool kVecOut>
+template <int P, int CL, bool kTMA, bool kVecOut, bool kEx = false>
 __global__ void __launch_bounds__(kThreads<P>, 2)
     sat_tile_kernel(const __grid_constant__ CUtensorMap map, const KParams p) {
   using C = Cfg<P>;
@@ -1376,7 +1449,7 @@ __global__ void __launch_bounds__(kThreads<P>, 2)
   } else if (warp >= kFirstLbWarp<P>) {
     lookback_warp<P, CL>(sm, p, warp - kFirstLbWarp<P>, rank, lane);
   } else {
-    compute_warp<P, CL, kVecOut>(sm, p, warp, lane);
+    compute_warp<P, CL, kVecOut, kEx>(sm, p, warp, lane);
   }
 #ifdef SAT_PROFILE
   __syncthreads();

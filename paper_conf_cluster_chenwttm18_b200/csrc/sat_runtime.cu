@@ -69,7 +69,7 @@ static EncodeTiledFn get_encode() {
 template <int P>
 static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
                            int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
-                           const void* carry_in, cudaStream_t stream) {
+                           const void* carry_in, cudaStream_t stream, const ExSpec* ex) {
   using C = Cfg<P>;
   const bool tma = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
                    getenv_int("SAT_FORCE_GENERIC", 0) == 0;
@@ -87,6 +87,8 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.total_bands = kp.bands_per_image * batch;
   kp.nchunks = (int32_t)((w + C::TW - 1) / C::TW);
   kp.carry_in = carry_in;
+  kp.out_cols = ex ? ex->out_cols : w;
+  kp.nval_bits = ex ? ex->nval_bits : 0;
   if (kp.total_bands * kp.nchunks > pl->max_tiles)
     return fail(SAT_ERR_INVALID_ARGUMENT, "problem needs %lld tiles, plan holds %lld",
                 (long long)(kp.total_bands * kp.nchunks), (long long)pl->max_tiles);
@@ -131,6 +133,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   if (pl->cluster > 0) CL = pl->cluster;
   const int cl_env = getenv_int("SAT_CLUSTER", 0);
   if (cl_env == 1 || cl_env == 4 || cl_env == 8) CL = cl_env;
+  if (ex && CL == 1) CL = 4;  // exclusive kernels are instantiated for clusters of 4 and 8
   const int ci = cluster_index(CL);
   kp.total_tickets = (kp.total_bands + CL - 1) / CL;
   // Persistent grid: every co-resident cluster slot, but no more clusters than tickets.
@@ -155,18 +158,20 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   cfg.numAttrs = 1;
   size_t smem = 0;
   cudaError_t e = cudaSuccess;
-#define SAT_LAUNCH_CL(CLV)                                                                  \
+#define SAT_LAUNCH_CL(CLV, EX)                                                              \
   {                                                                                         \
     smem = sizeof(Smem<P, CLV>);                                                            \
     cfg.dynamicSmemBytes = smem;                                                            \
     switch (mode) {                                                                         \
-      case 0: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, false, false>, map, kp); break; \
-      case 1: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, true, false>, map, kp); break;  \
-      case 2: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, false, true>, map, kp); break;  \
-      default: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, true, true>, map, kp); break;  \
+      case 0: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, false, false, EX>, map, kp); break; \
+      case 1: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, true, false, EX>, map, kp); break;  \
+      case 2: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, false, true, EX>, map, kp); break;  \
+      default: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, true, true, EX>, map, kp); break;  \
     }                                                                                       \
   }
-  if (CL == 1) SAT_LAUNCH_CL(1) else if (CL == 4) SAT_LAUNCH_CL(4) else SAT_LAUNCH_CL(8)
+  if (ex) {
+    if (CL == 4) SAT_LAUNCH_CL(4, true) else SAT_LAUNCH_CL(8, true)
+  } else if (CL == 1) SAT_LAUNCH_CL(1, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
 #undef SAT_LAUNCH_CL
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
   e = cudaGetLastError();
@@ -230,14 +235,14 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
 
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
-                  cudaStream_t stream) {
+                  cudaStream_t stream, const ExSpec* ex) {
   switch (pl->pair) {
     case SAT_8U_32S:
-      return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream);
+      return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
     case SAT_32F_32F:
-      return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream);
+      return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
     case SAT_64F_64F:
-      return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream);
+      return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
@@ -269,6 +274,15 @@ static sat_status configure_cl(sat_plan_st* pl) {
   cudaError_t e0 = cudaFuncSetAttribute(sat_occupancy_proxy<P, CL>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e0 != cudaSuccess) return cuda_fail(e0, "cudaFuncSetAttribute(proxy)");
+  if constexpr (CL != 1) {
+    void (*fx[4])(CUtensorMap, KParams) = {
+        sat_tile_kernel<P, CL, false, false, true>, sat_tile_kernel<P, CL, true, false, true>,
+        sat_tile_kernel<P, CL, false, true, true>, sat_tile_kernel<P, CL, true, true, true>};
+    for (int m = 0; m < 4; ++m) {
+      cudaError_t e = cudaFuncSetAttribute(fx[m], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(exclusive)");
+    }
+  }
   for (int m = 0; m < 4; ++m) {
     cudaError_t e = cudaFuncSetAttribute(fns[m], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
@@ -487,6 +501,81 @@ sat_status sat_compute_batched(sat_plan plan, const void* in, void* out, int64_t
                 batch > 1 ? in_image_stride_bytes : h * in_pitch_bytes,
                 batch > 1 ? out_image_stride_bytes : h * out_pitch_bytes, batch, nullptr,
                 static_cast<cudaStream_t>(stream));
+}
+
+}  // extern "C"
+
+namespace {
+// rows x cols block of one value (the exclusive layout's nVal border)
+template <typename T>
+__global__ void fill2d_kernel(char* out, int64_t rows, int64_t cols, int64_t pitch, T v) {
+  const int64_t n = rows * cols;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    reinterpret_cast<T*>(out + (i / cols) * pitch)[i % cols] = v;
+}
+
+sat_status fill2d(sat_pair pair, void* out, int64_t rows, int64_t cols, int64_t pitch,
+                  uint64_t bits, cudaStream_t s) {
+  if (rows <= 0 || cols <= 0) return SAT_OK;
+  const int64_t n = rows * cols;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 4096);
+  if (pair == SAT_64F_64F) {
+    double v;
+    memcpy(&v, &bits, 8);
+    fill2d_kernel<double><<<grid, 256, 0, s>>>((char*)out, rows, cols, pitch, v);
+  } else {
+    uint32_t v = (uint32_t)bits;
+    fill2d_kernel<uint32_t><<<grid, 256, 0, s>>>((char*)out, rows, cols, pitch, v);
+  }
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "fill2d_kernel launch");
+}
+}  // namespace
+
+extern "C" {
+
+sat_status sat_compute_exclusive(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                                 int64_t in_pitch_bytes, int64_t out_pitch_bytes, int full,
+                                 const void* nval, sat_pair pair, void* stream) {
+  if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (pair != plan->pair)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "pair %d does not match the plan's pair %d", (int)pair,
+                (int)plan->pair);
+  if (h < 0 || w < 0) return fail(SAT_ERR_INVALID_ARGUMENT, "negative extent");
+  if (full != 0 && full != 1) return fail(SAT_ERR_INVALID_ARGUMENT, "full must be 0 or 1");
+  const int64_t sa = (int64_t)in_size(pair), sb = (int64_t)out_size(pair);
+  const int64_t out_rows = full ? h + 1 : h, out_cols = full ? w + 1 : w;
+  if (out_rows == 0 || out_cols == 0) return SAT_OK;
+  if (!out) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL output pointer");
+  if (out_pitch_bytes < out_cols * sb || out_pitch_bytes % sb != 0 || (uintptr_t)out % sb != 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "output pitch %lld / alignment invalid for %lld columns",
+                (long long)out_pitch_bytes, (long long)out_cols);
+  uint64_t bits = 0;
+  if (nval) memcpy(&bits, nval, (size_t)sb);
+  const int64_t hk = full ? h : h - 1;  // input rows whose SAT lands in the output
+  if (hk > 0 && w > 0) {
+    if (!in) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL input pointer");
+    const size_t in_bytes = (size_t)((h - 1) * in_pitch_bytes + w * sa);
+    const size_t out_bytes = (size_t)((out_rows - 1) * out_pitch_bytes + out_cols * sb);
+    if (ranges_overlap(in, in_bytes, out, out_bytes))
+      return fail(SAT_ERR_UNSUPPORTED, "input and output overlap (exclusive layout is never in place)");
+  }
+  DeviceGuard g(plan->device);
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (hk <= 0 || w == 0) {  // border only: every element is nVal
+    return fill2d(pair, out, out_rows, out_cols, out_pitch_bytes, bits, s);
+  }
+  bool empty = false;
+  char* out1 = static_cast<char*>(out) + out_pitch_bytes;
+  sat_status st = validate(plan, in, out1, hk, w, in_pitch_bytes, out_pitch_bytes,
+                           hk * in_pitch_bytes, hk * out_pitch_bytes, 1, pair, &empty);
+  if (st != SAT_OK || empty) return st;
+  st = fill2d(pair, out, 1, out_cols, out_pitch_bytes, bits, s);  // row 0
+  if (st != SAT_OK) return st;
+  const ExSpec ex{out_cols, bits};
+  return launch(plan, in, out1, hk, w, in_pitch_bytes, out_pitch_bytes, hk * in_pitch_bytes,
+                hk * out_pitch_bytes, 1, nullptr, s, &ex);
 }
 
 sat_status sat_compute(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
