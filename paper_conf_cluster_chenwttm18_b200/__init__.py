@@ -231,7 +231,10 @@ def sat_exclusive(x, full: bool = True, nval=0, out=None, plan: Plan | None = No
     H, W = x.shape
     shape = (H + 1, W + 1) if full else (H, W)
     if out is None:
-        out = torch.empty(shape, dtype=out_dtype(pair), device=x.device)
+        # rows padded to 16 bytes (a view), so the kernel's shifted stores stay vectorised
+        per16 = 16 // torch.empty((), dtype=out_dtype(pair)).element_size()
+        cols = -(-max(shape[1], 1) // per16) * per16
+        out = torch.empty((shape[0], cols), dtype=out_dtype(pair), device=x.device)[:, :shape[1]]
     elif out.dtype != out_dtype(pair) or tuple(out.shape) != shape or out.device != x.device:
         raise ValueError("out has the wrong dtype/shape/device")
     if out.numel() == 0:

@@ -73,6 +73,12 @@ def main():
         ms = timeit(lambda: sat.sat(x, out=ours_out), steps, ws)
         res["entries"].append({"impl": "libsat sat_compute", "pair": "8u->32s", "shape": f"{H}x{W}",
                                "ms": ms, "gpx_s": px / ms / 1e6, "alg_gbs": ws / ms / 1e6})
+        # NPP-style pitched output (rows padded to 16 B, like nppiMalloc)
+        ex_out = torch.empty((H + 1, W + 4), dtype=torch.int32, device="cuda")[:, :W + 1]
+        ms = timeit(lambda: sat.sat_exclusive(x, full=True, out=ex_out), steps, ws)
+        res["entries"].append({"impl": "libsat sat_compute_exclusive (H+1)x(W+1)", "pair": "8u->32s",
+                               "shape": f"{H}x{W}", "ms": ms, "gpx_s": px / ms / 1e6,
+                               "alg_gbs": ws / ms / 1e6})
         if lib is not None:
             for name, dt, fn in (("nppiIntegral_8u32s_C1R", torch.int32, lib.nppiIntegral_8u32s_C1R),
                                  ("nppiIntegral_8u32f_C1R", torch.float32, lib.nppiIntegral_8u32f_C1R)):
@@ -93,6 +99,7 @@ def main():
                     # agreement with libsat on the interior (exclusive layout shifted by one)
                     if dt == torch.int32:
                         entry["matches_libsat"] = bool(torch.equal(o[1:, 1:], ours_out))
+                        entry["matches_libsat_exclusive"] = bool(torch.equal(o, ex_out))
                     ms = timeit(lambda: fn(x.data_ptr(), W, o.data_ptr(), (W + 1) * 4, NppiSize(W, H), nval),
                                 steps, ws)
                     entry.update({"ms": ms, "gpx_s": px / ms / 1e6, "alg_gbs": ws / ms / 1e6})
@@ -124,7 +131,7 @@ def main():
         res["entries"].append({"impl": "torch cumsum(0).cumsum(1) float32", "pair": "32f->32f",
                                "shape": f"{H}x{W}", "ms": ms, "gpx_s": px / ms / 1e6,
                                "alg_gbs": px * 8 / ms / 1e6})
-        del x, xf, of, ours_out
+        del x, xf, of, ours_out, ex_out
         torch.cuda.empty_cache()
     print(json.dumps(res))
 
