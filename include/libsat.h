@@ -138,6 +138,29 @@ sat_status sat_compute_exclusive(sat_plan plan, const void* in, void* out, int64
                                  const void* nval, sat_pair pair, void* stream);
 
 /* ---------------------------------------------------------------------------
+ * SAT consumers: O(1) rectangle sums from an
+ * inclusive SAT by the four-corner identity (motivation
+ * PAPER.md:18-24).  `sat` is a device SAT as written by sat_compute (T_B
+ * elements, sat_pitch_bytes per row).  For 8u->32s the SAT holds the sums
+ * mod 2^32 and so do the results: exact whenever the rectangle's true sum is
+ * below 2^32, even where the SAT itself wrapped. */
+
+/* n rectangle sums.  rects: device int32[n][4] = {y0, x0, y1, x1} (16-byte
+ * aligned), the half-open rectangle [y0, y1) x [x0, x1) of the image;
+ * coordinates are clamped to [0, h] / [0, w] and an empty rectangle sums to 0.
+ * out: device T_B[n]. */
+sat_status sat_rect_sums(sat_plan plan, const void* sat, int64_t h, int64_t w,
+                         int64_t sat_pitch_bytes, const void* rects, int64_t n, void* out,
+                         sat_pair pair, void* stream);
+
+/* Box filter (box sum): out(y, x) = sum of A over [y-ry, y+ry] x [x-rx, x+rx]
+ * clipped to the image, for every pixel; out is h x w of T_B (device, must not
+ * overlap the SAT).  ry, rx >= 0. */
+sat_status sat_box_filter(sat_plan plan, const void* sat, void* out, int64_t h, int64_t w,
+                          int64_t sat_pitch_bytes, int64_t out_pitch_bytes, int64_t ry,
+                          int64_t rx, sat_pair pair, void* stream);
+
+/* ---------------------------------------------------------------------------
  * Multi-GPU (one process per GPU, NCCL over NVLink/NVSwitch).
  * NCCL is loaded at run time (dlopen "libnccl.so.2"; the copy torch already
  * loaded is reused).  Errors from NCCL map to SAT_ERR_NCCL.

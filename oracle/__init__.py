@@ -167,3 +167,39 @@ def sat_exclusive_brute(A: np.ndarray, full: bool = True, nval=0) -> np.ndarray:
             else:
                 out[y, x] = float(s + Fraction(float(nval)))
     return out
+
+
+def rect_sums(A: np.ndarray, rects) -> np.ndarray:
+    """Direct sums of A over half-open rectangles [y0, y1) x [x0, x1) (clamped),
+    straight from the input -- the quantity the four-corner identity of
+    PAPER.md:95 recovers from a SAT.  8u: int64 sum reported mod 2^32 (int32)."""
+    H, W = A.shape
+    pair = pair_of(A)
+    out = []
+    for y0, x0, y1, x1 in np.asarray(rects, dtype=np.int64).reshape(-1, 4):
+        y0, y1 = min(max(y0, 0), H), min(max(y1, 0), H)
+        x0, x1 = min(max(x0, 0), W), min(max(x1, 0), W)
+        blk = A[y0:y1, x0:x1]
+        if pair == PAIR_8U32S:
+            v = int(blk.astype(np.int64).sum()) if y1 > y0 and x1 > x0 else 0
+            out.append(np.uint32(v & 0xFFFFFFFF).view(np.int32))
+        else:
+            out.append(float(blk.astype(np.float64).sum()) if y1 > y0 and x1 > x0 else 0.0)
+    return np.array(out, dtype=np.int32 if pair == PAIR_8U32S else np.float64)
+
+
+def box_filter(A: np.ndarray, ry: int, rx: int) -> np.ndarray:
+    """Box sums out(y, x) = sum of A over [y-ry, y+ry] x [x-rx, x+rx] clipped to
+    the image, as a sum of shifted copies of the zero-padded input (no SAT
+    involved).  8u: exact int64, reported mod 2^32; floats: fp64."""
+    H, W = A.shape
+    pair = pair_of(A)
+    P = np.zeros((H + 2 * ry, W + 2 * rx), dtype=np.int64 if pair == PAIR_8U32S else np.float64)
+    P[ry:ry + H, rx:rx + W] = A
+    out = np.zeros((H, W), dtype=P.dtype)
+    for dy in range(2 * ry + 1):
+        for dx in range(2 * rx + 1):
+            out += P[dy:dy + H, dx:dx + W]
+    if pair == PAIR_8U32S:
+        return (out & 0xFFFFFFFF).astype(np.uint32).view(np.int32)
+    return out

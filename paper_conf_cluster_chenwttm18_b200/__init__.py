@@ -58,6 +58,8 @@ def lib():
                     "sat_compute_band": ([vp, vp, vp, i64, i64, i64, i64, vp, i32, vp], i32),
                     "sat_compute_host": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_exclusive": ([vp, vp, vp, i64, i64, i64, i64, i32, vp, i32, vp], i32),
+                    "sat_rect_sums": ([vp, vp, i64, i64, i64, vp, i64, vp, i32, vp], i32),
+                    "sat_box_filter": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i32, vp], i32),
                     "sat_comm_unique_id": ([vp], i32),
                     "sat_comm_create": ([ctypes.POINTER(vp), vp, i32, i32, i32], i32),
                     "sat_comm_destroy": ([vp], i32),
@@ -248,6 +250,43 @@ def sat_exclusive(x, full: bool = True, nval=0, out=None, plan: Plan | None = No
                                        out.data_ptr(), H, W, ip, op, 1 if full else 0,
                                        ctypes.byref(nv), pair, _stream_ptr(stream, x.device)),
            "sat_compute_exclusive")
+    return out
+
+
+def rect_sums(S, rects, plan: Plan | None = None, stream=None):
+    """Sums of A over half-open rectangles [y0, y1) x [x0, x1) from its inclusive
+    SAT S (a CUDA tensor as returned by sat()); rects: int32 CUDA tensor [n, 4]
+    of (y0, x0, y1, x1), clamped to the image."""
+    torch = _torch()
+    pair = {torch.int32: 0, torch.float32: 1, torch.float64: 2}[S.dtype]
+    H, W = S.shape
+    rects = rects.to(device=S.device, dtype=torch.int32).contiguous()
+    if rects.dim() != 2 or rects.shape[1] != 4:
+        raise ValueError("rects must be [n, 4]")
+    out = torch.empty(rects.shape[0], dtype=S.dtype, device=S.device)
+    if rects.shape[0] == 0:
+        return out
+    sp = _row_layout(S)[0] if H > 0 and W > 0 else max(W, 1) * S.element_size()
+    p = plan if plan is not None else _plan_for(S.device, pair, max(H, 1), max(W, 1), 1)
+    _check(lib().sat_rect_sums(p.handle, S.data_ptr() if S.numel() else None, H, W, sp,
+                               rects.data_ptr(), rects.shape[0], out.data_ptr(), pair,
+                               _stream_ptr(stream, S.device)), "sat_rect_sums")
+    return out
+
+
+def box_filter(S, ry: int, rx: int, out=None, plan: Plan | None = None, stream=None):
+    """Box sums of radius (ry, rx), clipped at the borders, from the inclusive SAT S."""
+    torch = _torch()
+    pair = {torch.int32: 0, torch.float32: 1, torch.float64: 2}[S.dtype]
+    H, W = S.shape
+    if out is None:
+        out = torch.empty((H, W), dtype=S.dtype, device=S.device)
+    if H == 0 or W == 0:
+        return out
+    p = plan if plan is not None else _plan_for(S.device, pair, H, W, 1)
+    _check(lib().sat_box_filter(p.handle, S.data_ptr(), out.data_ptr(), H, W, _row_layout(S)[0],
+                                _row_layout(out)[0], ry, rx, pair, _stream_ptr(stream, S.device)),
+           "sat_box_filter")
     return out
 
 

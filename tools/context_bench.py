@@ -73,6 +73,19 @@ def main():
         ms = timeit(lambda: sat.sat(x, out=ours_out), steps, ws)
         res["entries"].append({"impl": "libsat sat_compute", "pair": "8u->32s", "shape": f"{H}x{W}",
                                "ms": ms, "gpx_s": px / ms / 1e6, "alg_gbs": ws / ms / 1e6})
+        # SAT consumers (N4): box sums of radius 8 from the SAT (reads S, writes out: 8 B/px)
+        bo = torch.empty((H, W), dtype=torch.int32, device="cuda")
+        ms = timeit(lambda: sat.box_filter(ours_out, 8, 8, out=bo), steps, px * 8)
+        res["entries"].append({"impl": "libsat sat_box_filter r=8 (from SAT)", "pair": "32s->32s",
+                               "shape": f"{H}x{W}", "ms": ms, "gpx_s": px / ms / 1e6,
+                               "alg_gbs": px * 8 / ms / 1e6})
+        del bo
+        nq = 1 << 22
+        rq = torch.randint(0, min(H, W), (nq, 4), dtype=torch.int32, device="cuda")
+        ms = timeit(lambda: sat.rect_sums(ours_out, rq), steps, nq * 20)
+        res["entries"].append({"impl": "libsat sat_rect_sums 4M random rects", "pair": "32s",
+                               "shape": f"{H}x{W}", "ms": ms, "gqueries_s": nq / ms / 1e6})
+        del rq
         # NPP-style pitched output (rows padded to 16 B, like nppiMalloc)
         ex_out = torch.empty((H + 1, W + 4), dtype=torch.int32, device="cuda")[:, :W + 1]
         ms = timeit(lambda: sat.sat_exclusive(x, full=True, out=ex_out), steps, ws)
