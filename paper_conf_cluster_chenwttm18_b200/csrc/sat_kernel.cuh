@@ -77,7 +77,6 @@ struct Cfg<P8U32S> {
   static constexpr int E = 4;   // consecutive elements per lane-group (16 B out)
   static constexpr int G = 2;   // groups per lane: cols {4l..4l+3} and {128+4l..}
   static constexpr int TW = 32 * E * G;  // 256
-  static constexpr int TH = 32;
 #ifndef SAT_LOOK8
 #define SAT_LOOK8 3
 #endif
@@ -85,8 +84,9 @@ struct Cfg<P8U32S> {
 #ifndef SAT_NCW8
 #define SAT_NCW8 8
 #endif
-  static constexpr int NCW = SAT_NCW8;   // compute warps (TH / NCW rows each)
-  static constexpr int NSTAGE = NCW > 8 ? 3 : 4;  // TMA prefetch depth (stages free after pass A)
+  static constexpr int NCW = SAT_NCW8;   // compute warps, 4 rows each
+  static constexpr int TH = 4 * NCW;     // 32 (2 CTAs per SM) or 64 (1 CTA per SM, 16 warps)
+  static constexpr int NSTAGE = 4;       // TMA prefetch depth (stages free after pass A)
 };
 template <>
 struct Cfg<P32F32F> {
@@ -148,12 +148,17 @@ constexpr int kNTot = (Cfg<P>::LOOK + 1 > kNLB) ? Cfg<P>::LOOK + 1 : kNLB;  // >
 template <int P>
 constexpr int kTmemColsPerWarp =
     (Cfg<P>::TH / kNCW<P>) * Cfg<P>::G * Cfg<P>::E * (int)(sizeof(typename Cfg<P>::TB) / 4);
-constexpr int kTmemCols = 256;  // per CTA (2 CTAs per SM share the SM's 512 columns)
+// TMEM columns per CTA: 8 compute warps -> 256 (2 CTAs per SM share the SM's
+// 512 columns); 16 compute warps -> 512 (one CTA per SM).
+template <int P>
+constexpr int kTmemCols = 256 * Cfg<P>::NCW / 8;
+template <int P>
+constexpr int kMinBlocks = Cfg<P>::NCW > 8 ? 1 : 2;  // resident CTAs per SM
 template <int P>
 constexpr int kTmemColsPerSlot = kTmemColsPerWarp<P> * (kNCW<P> / 4);  // NCW/4 warps per subpartition
-static_assert(kTmemColsPerSlot<P8U32S> * kNTot<P8U32S> <= kTmemCols, "TMEM budget (8u)");
-static_assert(kTmemColsPerSlot<P32F32F> * kNTot<P32F32F> <= kTmemCols, "TMEM budget (32f)");
-static_assert(kTmemColsPerSlot<P64F64F> * kNTot<P64F64F> <= kTmemCols, "TMEM budget (64f)");
+static_assert(kTmemColsPerSlot<P8U32S> * kNTot<P8U32S> <= kTmemCols<P8U32S>, "TMEM budget (8u)");
+static_assert(kTmemColsPerSlot<P32F32F> * kNTot<P32F32F> <= kTmemCols<P32F32F>, "TMEM budget (32f)");
+static_assert(kTmemColsPerSlot<P64F64F> * kNTot<P64F64F> <= kTmemCols<P64F64F>, "TMEM budget (64f)");
 
 struct KParams {
   const char* in;       // generic-path input base (TMA path uses the tensor map)
@@ -1395,7 +1400,7 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
 // ---------------------------------------------------------------------------
 
 template <int P, int CL, bool kTMA, bool kVecOut, bool kEx = false>
-__global__ void __launch_bounds__(kThreads<P>, 2)
+__global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
     sat_tile_kernel(const __grid_constant__ CUtensorMap map, const KParams p) {
   using C = Cfg<P>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -1429,7 +1434,7 @@ __global__ void __launch_bounds__(kThreads<P>, 2)
   if (warp == 0) {  // TMEM for the S' rows (one warp allocates and later frees)
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                      smem_u32(&sm.tmem_base)),
-                 "r"(kTmemCols)
+                 "r"(kTmemCols<P>)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
@@ -1464,7 +1469,7 @@ __global__ void __launch_bounds__(kThreads<P>, 2)
   if (warp == 0) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(sm.tmem_base),
-                 "r"(kTmemCols)
+                 "r"(kTmemCols<P>)
                  : "memory");
   }
 }

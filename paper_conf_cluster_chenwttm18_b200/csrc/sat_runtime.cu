@@ -260,7 +260,7 @@ int getenv_int(const char* name, int dflt) {
 // block size, dynamic shared memory, cluster shape and register bound, so its
 // answer is the real residency, which is then capped by TMEM.
 template <int P, int CL>
-__global__ void __launch_bounds__(kThreads<P>, 2) sat_occupancy_proxy(int* sink) {
+__global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>) sat_occupancy_proxy(int* sink) {
   extern __shared__ unsigned char s[];
   if (sink) sink[threadIdx.x] = s[threadIdx.x];
 }
@@ -300,7 +300,7 @@ static sat_status configure_cl(sat_plan_st* pl) {
     int n = 0;
     e = cudaOccupancyMaxActiveClusters(&n, sat_occupancy_proxy<P, CL>, &cfg);
     if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
-    const int tmem_cap = pl->num_sms * (512 / kTmemCols) / CL;
+    const int tmem_cap = pl->num_sms * (512 / kTmemCols<P>) / CL;
     pl->active_clusters[P][cluster_index(CL)][m] = std::min(n, tmem_cap);
   }
   return SAT_OK;
