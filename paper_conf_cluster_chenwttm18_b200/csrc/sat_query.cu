@@ -84,9 +84,75 @@ __global__ void __launch_bounds__(256) box_kernel(const char* sat, int64_t sp, c
   }
 }
 
+// Tiled box filter: a block stages the SAT window its 32 x 256 output tile
+// needs -- (32 + 2ry + 1) x (256 + 2rx + 1) elements, read once with
+// coalesced rows -- in shared memory, then every thread walks one output
+// column down the tile with four shared-memory corner reads per output.
+// Staged element (r, c) is S(min(ya + r, h - 1), min(xa + c, w - 1)) with
+// ya = y_tile - ry - 1, xa = x_tile - rx - 1, and 0 where ya + r < 0 or
+// xa + c < 0: exactly the clipped corners of the four-corner identity.
+constexpr int kBoxRows = 32, kBoxCols = 256;
+
+template <typename T>
+__global__ void __launch_bounds__(kBoxCols) box_tiled_kernel(const char* sat, int64_t sp, char* out,
+                                                             int64_t op, int64_t h, int64_t w,
+                                                             int ry, int rx) {
+  using A = typename Acc<T>::type;
+  extern __shared__ __align__(16) unsigned char box_smem[];
+  A* tile = reinterpret_cast<A*>(box_smem);
+  const int R = kBoxRows + 2 * ry + 1, C = kBoxCols + 2 * rx + 1;
+  const int64_t yt = (int64_t)blockIdx.y * kBoxRows, xt = (int64_t)blockIdx.x * kBoxCols;
+  const int64_t ya = yt - ry - 1, xa = xt - rx - 1;
+  // staging: 8 independent row loads in flight per thread before the smem stores
+  for (int c = threadIdx.x; c < C; c += kBoxCols) {
+    const int64_t x = xa + c;
+    const int64_t xc = std::min<int64_t>(x, w - 1);
+    for (int r0 = 0; r0 < R; r0 += 8) {
+      A v[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int64_t y = ya + r0 + k;
+        v[k] = (r0 + k >= R || y < 0 || x < 0)
+                   ? A(0)
+                   : (A)__ldg(reinterpret_cast<const T*>(sat + std::min<int64_t>(y, h - 1) * sp) + xc);
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k)
+        if (r0 + k < R) tile[(r0 + k) * C + c] = v[k];
+    }
+  }
+  __syncthreads();
+  const int tx = threadIdx.x;
+  const int64_t x = xt + tx;
+  if (x >= w) return;
+  const int dy = 2 * ry + 1, dx = 2 * rx + 1;
+  for (int ty = 0; ty < kBoxRows; ++ty) {
+    const int64_t y = yt + ty;
+    if (y >= h) break;
+    const A* top = tile + ty * C + tx;
+    const A* bot = top + dy * C;
+    reinterpret_cast<T*>(out + y * op)[x] = (T)((bot[dx] - top[dx]) - (bot[0] - top[0]));
+  }
+}
+
 template <typename T>
 sat_status launch_box(const void* sat, void* out, int64_t h, int64_t w, int64_t sp, int64_t op,
                       int64_t ry, int64_t rx, cudaStream_t s) {
+  const int64_t smem = (kBoxRows + 2 * ry + 1) * (kBoxCols + 2 * rx + 1) * (int64_t)sizeof(T);
+  if (smem <= 200 * 1024) {
+    static bool attr_set = false;  // per instantiation; benign race (idempotent)
+    if (!attr_set) {
+      cudaError_t e = cudaFuncSetAttribute(box_tiled_kernel<T>,
+                                           cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+      if (e != cudaSuccess) return sat::cuda_fail(e, "cudaFuncSetAttribute(box_tiled_kernel)");
+      attr_set = true;
+    }
+    dim3 grid((unsigned)((w + kBoxCols - 1) / kBoxCols), (unsigned)((h + kBoxRows - 1) / kBoxRows));
+    box_tiled_kernel<T><<<grid, kBoxCols, (size_t)smem, s>>>(
+        static_cast<const char*>(sat), sp, static_cast<char*>(out), op, h, w, (int)ry, (int)rx);
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? SAT_OK : sat::cuda_fail(e, "box_tiled_kernel launch");
+  }
   constexpr int ROWS = 64;
   dim3 grid((unsigned)((w + 31) / 32), (unsigned)((h + ROWS - 1) / ROWS));
   box_kernel<T, ROWS><<<grid, dim3(32, 8), 0, s>>>(static_cast<const char*>(sat), sp,
