@@ -17,6 +17,7 @@ struct sat_plan_st {
   int64_t max_h = 0, max_w = 0, max_batch = 0;
   int num_sms = 0;
   int active_clusters[3][3][4] = {};  // [pair][cluster 1/4/8][mode: bit0 TMA, bit1 vec out]
+  int active_short[3] = {};           // [pair] short-band variant, clusters of 4, TMA + vec out
   int cluster = 0;                    // forced CTAs (bands) per cluster (0: by shape)
   int64_t max_tiles = 0;       // capacity of the look-back workspace in tiles
   void* ws = nullptr;

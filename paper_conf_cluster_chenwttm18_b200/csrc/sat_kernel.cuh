@@ -58,6 +58,12 @@
 namespace sat {
 
 enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2 };
+// Short-band variants (P + kShort): the same pair with 16-row bands (2 rows per
+// compute warp), chosen for short, wide images whose 32-row bands would leave
+// most of the machine idle (H / 4 compute warps in total otherwise).
+constexpr int kShort = 3;
+template <int P>
+constexpr int kBase = P % kShort;
 
 #ifndef SAT_NLB
 #define SAT_NLB 3
@@ -118,6 +124,17 @@ struct Cfg<P64F64F> {
   static constexpr int NCW = 8;
   static constexpr int NSTAGE = 3;
 };
+template <int P>
+struct CfgShort : Cfg<P> {
+  static constexpr int TH = Cfg<P>::TH / 2;
+};
+template <>
+struct Cfg<P8U32S + kShort> : CfgShort<P8U32S> {};
+template <>
+struct Cfg<P32F32F + kShort> : CfgShort<P32F32F> {};
+template <>
+struct Cfg<P64F64F + kShort> : CfgShort<P64F64F> {};
+
 
 // Warp roles: NCW compute warps, then the producer, then kNLB look-back warps.
 template <int P>
@@ -468,6 +485,20 @@ __device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&v)[32]) {
       : "r"(taddr)
       : "memory");
 }
+__device__ __forceinline__ void tmem_st(uint32_t taddr, const uint32_t (&v)[8]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&v)[8]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]),
+        "=r"(v[7])
+      : "r"(taddr)
+      : "memory");
+}
 __device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, "
@@ -722,7 +753,7 @@ __device__ __forceinline__ void publish(const KParams& p, int64_t T, int32_t chu
 #pragma unroll
   for (int g = 0; g < C::G; ++g) {
     uint64_t w[4];
-    Tag<P>::enc(v[g], (p.epoch << 2) | st, w);
+    Tag<kBase<P>>::enc(v[g], (p.epoch << 2) | st, w);
     uint64_t* dst = row + (g * 32 + lane) * 4;
     st_relaxed_v2_u64(dst, w[0], w[1]);
     st_relaxed_v2_u64(dst + 2, w[2], w[3]);
@@ -815,7 +846,7 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
 #pragma unroll
         for (int e = 0; e < 4; ++e) w[e] = land[b][(g * 32 + lane) * 4 + e];
         TB t[C::E];
-        Tag<P>::dec(w, t);
+        Tag<kBase<P>>::dec(w, t);
 #pragma unroll
         for (int e = 0; e < C::E; ++e) V[g][e] += t[e];
       }

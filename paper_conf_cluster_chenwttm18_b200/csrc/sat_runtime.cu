@@ -89,7 +89,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.carry_in = carry_in;
   kp.out_cols = ex ? ex->out_cols : w;
   kp.nval_bits = ex ? ex->nval_bits : 0;
-  if (kp.total_bands * kp.nchunks > pl->max_tiles)
+  if ((kp.total_bands + (P >= kShort ? 1 : 0)) / (P >= kShort ? 2 : 1) * kp.nchunks > pl->max_tiles)
     return fail(SAT_ERR_INVALID_ARGUMENT, "problem needs %lld tiles, plan holds %lld",
                 (long long)(kp.total_bands * kp.nchunks), (long long)pl->max_tiles);
 
@@ -98,8 +98,8 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   if (tma) {
     EncodeTiledFn enc = get_encode();
     if (!enc) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
-    const CUtensorMapDataType dt = P == P8U32S    ? CU_TENSOR_MAP_DATA_TYPE_UINT8
-                                   : P == P32F32F ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+    const CUtensorMapDataType dt = kBase<P> == P8U32S    ? CU_TENSOR_MAP_DATA_TYPE_UINT8
+                                   : kBase<P> == P32F32F ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
                                                   : CU_TENSOR_MAP_DATA_TYPE_FLOAT64;
     cuuint64_t dims[3] = {(cuuint64_t)w, (cuuint64_t)h, (cuuint64_t)batch};
     cuuint64_t strides[2] = {(cuuint64_t)ip, (cuuint64_t)(batch > 1 ? iis : ip * h)};
@@ -129,15 +129,17 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   // bands to fill the machine (shorter look-back chains pay off there); 4 for
   // 8u->32s and for short/wide images (measured).
   const int64_t nbands = kp.total_bands;
-  int CL = (P != P8U32S && nbands >= 264) ? 8 : 4;
+  int CL = (kBase<P> != P8U32S && nbands >= 264) ? 8 : 4;
   if (pl->cluster > 0) CL = pl->cluster;
   const int cl_env = getenv_int("SAT_CLUSTER", 0);
   if (cl_env == 1 || cl_env == 4 || cl_env == 8) CL = cl_env;
   if (ex && CL == 1) CL = 4;  // exclusive kernels are instantiated for clusters of 4 and 8
+  if (P >= kShort) CL = 4;    // short-band kernels: clusters of 4 only
   const int ci = cluster_index(CL);
   kp.total_tickets = (kp.total_bands + CL - 1) / CL;
   // Persistent grid: every co-resident cluster slot, but no more clusters than tickets.
-  int64_t clusters = std::max(pl->active_clusters[P][ci][mode], 1);
+  int64_t clusters =
+      std::max(P >= kShort ? pl->active_short[kBase<P>] : pl->active_clusters[kBase<P>][ci][mode], 1);
   const int cap = getenv_int("SAT_MAX_CLUSTERS", 0);
   if (cap > 0) clusters = std::min<int64_t>(clusters, cap);
   const int force = getenv_int("SAT_FORCE_CLUSTERS", 0);
@@ -169,7 +171,11 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
       default: e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, CLV, true, true, EX>, map, kp); break;  \
     }                                                                                       \
   }
-  if (ex) {
+  if constexpr (P >= kShort) {  // selected only for TMA + vector-store launches
+    smem = sizeof(Smem<P, 4>);
+    cfg.dynamicSmemBytes = smem;
+    e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, 4, true, true, false>, map, kp);
+  } else if (ex) {
     if (CL == 4) SAT_LAUNCH_CL(4, true) else SAT_LAUNCH_CL(8, true)
   } else if (CL == 1) SAT_LAUNCH_CL(1, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
 #undef SAT_LAUNCH_CL
@@ -236,6 +242,27 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
                   cudaStream_t stream, const ExSpec* ex) {
+  // Short, wide images: 32-row bands give only H/4 compute warps in total
+  // (2 CTAs of 8 warps per SM leave most SMs idle below ~140 bands); 16-row
+  // bands (2 rows per warp) double the warps in flight.
+  const int th = tile_h(pl->pair);
+  const int64_t bands32 = (h + th - 1) / th * batch;
+  const bool aligned = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
+                       ((uintptr_t)out % 16 == 0) && (op % 16 == 0) && (batch == 1 || ois % 16 == 0);
+  const int sh_env = getenv_int("SAT_SHORT", -1);
+  const bool use_short = !ex && aligned && getenv_int("SAT_FORCE_GENERIC", 0) == 0 &&
+                         getenv_int("SAT_CLUSTER", 0) == 0 && pl->cluster == 0 &&
+                         (sh_env >= 0 ? sh_env == 1 : 2 * bands32 <= (int64_t)pl->num_sms);
+  if (use_short) {
+    switch (pl->pair) {
+      case SAT_8U_32S:
+        return launch_t<P8U32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+      case SAT_32F_32F:
+        return launch_t<P32F32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+      case SAT_64F_64F:
+        return launch_t<P64F64F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+    }
+  }
   switch (pl->pair) {
     case SAT_8U_32S:
       return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
@@ -307,10 +334,39 @@ static sat_status configure_cl(sat_plan_st* pl) {
 }
 
 template <int P>
+static sat_status configure_short(sat_plan_st* pl) {
+  constexpr int PS = P + kShort, CL = 4;
+  const size_t smem = sizeof(Smem<PS, CL>);
+  cudaError_t e = cudaFuncSetAttribute(sat_occupancy_proxy<PS, CL>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sat_tile_kernel<PS, CL, true, true, false>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(short)");
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(CL * 64);
+  cfg.blockDim = dim3(kThreads<PS>);
+  cfg.dynamicSmemBytes = smem;
+  cudaLaunchAttribute attr;
+  attr.id = cudaLaunchAttributeClusterDimension;
+  attr.val.clusterDim.x = CL;
+  attr.val.clusterDim.y = 1;
+  attr.val.clusterDim.z = 1;
+  cfg.attrs = &attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  e = cudaOccupancyMaxActiveClusters(&n, sat_occupancy_proxy<PS, CL>, &cfg);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters(short)");
+  pl->active_short[P] = std::min(n, pl->num_sms * (512 / kTmemCols<PS>) / CL);
+  return SAT_OK;
+}
+
+template <int P>
 static sat_status configure_t(sat_plan_st* pl) {
   sat_status st = configure_cl<P, 1>(pl);
   if (st == SAT_OK) st = configure_cl<P, 4>(pl);
   if (st == SAT_OK) st = configure_cl<P, 8>(pl);
+  if (st == SAT_OK) st = configure_short<P>(pl);
   return st;
 }
 

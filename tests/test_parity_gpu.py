@@ -378,3 +378,38 @@ def test_generic_load_path_forced(monkeypatch, np_dtype):
     y = sat.sat(x)
     torch.cuda.synchronize()
     check(y.cpu().numpy(), oracle.sat(x.cpu().numpy()), np_dtype, "generic")
+
+
+@pytest.mark.parametrize("short", ["0", "1"])
+@pytest.mark.parametrize("np_dtype", [np.uint8, np.float32, np.float64])
+@pytest.mark.parametrize("shape", [(1, 1), (15, 300), (17, 257), (999, 1001), (2048, 4100)])
+def test_parity_short_bands(monkeypatch, short, np_dtype, shape):
+    """16-row-band kernels (chosen automatically for short, wide images)
+    forced on and off for every shape."""
+    torch = _torch()
+    sat = _sat()
+    monkeypatch.setenv("SAT_SHORT", short)
+    H, W = shape
+    x = gen(np_dtype, H, W, seed=2101 + H)
+    y = sat.sat(x)
+    torch.cuda.synchronize()
+    check(y.cpu().numpy(), oracle.sat(x.cpu().numpy()), np_dtype, f"short={short} {shape}")
+
+
+def test_short_bands_batched_and_carry(monkeypatch):
+    """Short-band kernels with batches straddled by clusters and with a band carry-in."""
+    torch = _torch()
+    sat = _sat()
+    monkeypatch.setenv("SAT_SHORT", "1")
+    x = torch.empty((9, 37, 1920), dtype=torch.uint8, device="cuda")
+    satgen.fill_device(x, seed=2201)
+    y = sat.sat(x)
+    torch.cuda.synchronize()
+    xs = x.cpu().numpy()
+    for i in range(9):
+        check(y[i].cpu().numpy(), oracle.sat(xs[i]), np.uint8, f"frame {i}")
+    full = gen(np.float64, 200, 700, seed=2202)
+    top = sat.sat(full[:77])
+    band = sat.sat_band(full[77:], carry_in=top[-1].contiguous())
+    torch.cuda.synchronize()
+    check(band.cpu().numpy(), oracle.sat(full.cpu().numpy())[77:], np.float64, "band carry")
