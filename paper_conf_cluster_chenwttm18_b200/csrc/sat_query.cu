@@ -140,13 +140,10 @@ sat_status launch_box(const void* sat, void* out, int64_t h, int64_t w, int64_t 
                       int64_t ry, int64_t rx, cudaStream_t s) {
   const int64_t smem = (kBoxRows + 2 * ry + 1) * (kBoxCols + 2 * rx + 1) * (int64_t)sizeof(T);
   if (smem <= 200 * 1024) {
-    static bool attr_set = false;  // per instantiation; benign race (idempotent)
-    if (!attr_set) {
-      cudaError_t e = cudaFuncSetAttribute(box_tiled_kernel<T>,
-                                           cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-      if (e != cudaSuccess) return sat::cuda_fail(e, "cudaFuncSetAttribute(box_tiled_kernel)");
-      attr_set = true;
-    }
+    // per device and cheap: set on every launch (a process may drive several GPUs)
+    cudaError_t ea = cudaFuncSetAttribute(box_tiled_kernel<T>,
+                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (ea != cudaSuccess) return sat::cuda_fail(ea, "cudaFuncSetAttribute(box_tiled_kernel)");
     dim3 grid((unsigned)((w + kBoxCols - 1) / kBoxCols), (unsigned)((h + kBoxRows - 1) / kBoxRows));
     box_tiled_kernel<T><<<grid, kBoxCols, (size_t)smem, s>>>(
         static_cast<const char*>(sat), sp, static_cast<char*>(out), op, h, w, (int)ry, (int)rx);

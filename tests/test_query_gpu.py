@@ -107,3 +107,36 @@ def test_box_filter_full_size_sampled_rows():
         blk = x[lo:hi].cpu().numpy()
         ref = oracle.box_filter(blk, ry, rx)[y - lo]
         assert np.array_equal(B[y].cpu().numpy(), ref), f"row {y}"
+
+
+def test_invalid_arguments_of_consumers_and_exclusive():
+    """sat_compute_exclusive / sat_rect_sums / sat_box_filter validate
+    synchronously and launch nothing on failure (libsat.h conventions)."""
+    import ctypes
+    torch, sat = _t(), _sat()
+    L = sat.lib()
+    x = torch.zeros((64, 64), dtype=torch.uint8, device="cuda")
+    S = torch.zeros((64, 64), dtype=torch.int32, device="cuda")
+    out = torch.full((65, 68), 5, dtype=torch.int32, device="cuda")
+    p = sat.Plan(0, 64, 64, 1)
+    h = p.handle
+    nv = ctypes.c_int32(1)
+    rects = torch.zeros((4, 4), dtype=torch.int32, device="cuda")
+    qo = torch.full((4,), 5, dtype=torch.int32, device="cuda")
+    cases = [
+        (L.sat_compute_exclusive(h, x.data_ptr(), out.data_ptr(), 64, 64, 64, 64 * 4, 1, ctypes.byref(nv), 0, None), 1),  # pitch < (w+1)*4
+        (L.sat_compute_exclusive(h, x.data_ptr(), out.data_ptr(), 64, 64, 64, 272, 2, ctypes.byref(nv), 0, None), 1),    # full not 0/1
+        (L.sat_compute_exclusive(h, x.data_ptr(), out.data_ptr(), 64, 64, 64, 272, 1, ctypes.byref(nv), 1, None), 1),    # pair
+        (L.sat_compute_exclusive(h, x.data_ptr(), x.data_ptr(), 16, 16, 64, 256, 1, None, 0, None), 2),                  # overlap
+        (L.sat_rect_sums(h, S.data_ptr(), 64, 64, 255, rects.data_ptr(), 4, qo.data_ptr(), 0, None), 1),                  # sat pitch
+        (L.sat_rect_sums(h, S.data_ptr(), 64, 64, 256, rects.data_ptr(), -1, qo.data_ptr(), 0, None), 1),                 # n < 0
+        (L.sat_rect_sums(h, S.data_ptr(), 64, 64, 256, rects.data_ptr() + 4, 4, qo.data_ptr(), 0, None), 1),              # misaligned rects
+        (L.sat_box_filter(h, S.data_ptr(), out.data_ptr(), 64, 64, 256, 272, -1, 2, 0, None), 1),                         # radius
+        (L.sat_box_filter(h, S.data_ptr(), S.data_ptr(), 64, 64, 256, 256, 1, 1, 0, None), 2),                            # overlap
+        (L.sat_box_filter(h, S.data_ptr(), out.data_ptr(), 64, 64, 256, 272, 1, 1, 2, None), 1),                          # pair
+    ]
+    for i, (got, want) in enumerate(cases):
+        assert got == want, f"case {i}: status {got}, want {want}"
+    torch.cuda.synchronize()
+    assert bool((out == 5).all()) and bool((qo == 5).all())
+    p.close()
