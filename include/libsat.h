@@ -191,6 +191,41 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
                             int64_t band_h, int64_t w, int64_t in_pitch_bytes,
                             int64_t out_pitch_bytes, sat_pair pair, void* stream);
 
+/* ---------------------------------------------------------------------------
+ * Chained row bands: the single-pass multi-GPU path.
+ * Instead of a column-sum pre-pass and an all-gather, each band's kernel
+ * publishes its bottom row S(r1-1, .) chunk by chunk (epoch-tagged 64-bit
+ * words, the look-back payload format) straight into the receive buffer of
+ * the band below -- on another GPU through peer memory -- whose top clusters
+ * wait for each chunk's vector as their look-back predecessor.  Bands are read
+ * once and written once (sizeof(T_A) + sizeof(T_B) bytes per pixel), and the
+ * bands overlap chunk by chunk. */
+
+/* Bytes of one chain buffer (the tagged carry vectors of one row of width w). */
+size_t sat_chain_bytes(sat_pair pair, int64_t w);
+
+/* One band of a chain on this device.  chain_in (NULL for the top band) is
+ * read, chain_out (NULL for the bottom band) is written: device or
+ * peer-mapped pointers, 16-byte aligned, sat_chain_bytes(pair, w) bytes,
+ * zero-filled once before first use.  chain_epoch in [1, 2^30) must differ
+ * from the previous use of the same buffer.  The band ABOVE must be able to
+ * run concurrently or earlier (e.g. same stream, earlier): a band waits in
+ * its kernel for chain_in.  h, w >= 1. */
+sat_status sat_compute_band_chained(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                                    int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                                    const void* chain_in, void* chain_out, uint32_t chain_epoch,
+                                    sat_pair pair, void* stream);
+
+/* Collective: rank r holds rows [sum_{r'<r} band_h_r', +band_h) (every band
+ * >= 1 row).  Receive buffers are exchanged once per width (CUDA IPC handles
+ * all-gathered over NCCL; needs peer access, i.e. NVLink between the GPUs);
+ * each call then does a one-int NCCL all-gather as a stream barrier (so no
+ * rank overwrites a buffer its peer still reads) and ONE kernel per rank. */
+sat_status sat_compute_dist_chained(sat_plan plan, sat_comm comm, const void* in_band,
+                                    void* out_band, int64_t band_h, int64_t w,
+                                    int64_t in_pitch_bytes, int64_t out_pitch_bytes, sat_pair pair,
+                                    void* stream);
+
 /* Building blocks of sat_compute_dist (steps 1 and 3), exported so the carry
  * algebra can be exercised without NCCL (e.g. "virtual ranks" on one GPU).
  * Accumulator type: uint32 for SAT_8U_32S (exact mod 2^32), double

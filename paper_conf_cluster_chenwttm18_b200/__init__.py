@@ -59,6 +59,9 @@ def lib():
                     "sat_compute_host": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_exclusive": ([vp, vp, vp, i64, i64, i64, i64, i32, vp, i32, vp], i32),
                     "sat_rect_sums": ([vp, vp, i64, i64, i64, vp, i64, vp, i32, vp], i32),
+                    "sat_chain_bytes": ([i32, i64], sz),
+                    "sat_compute_band_chained": ([vp, vp, vp, i64, i64, i64, i64, vp, vp, ctypes.c_uint32, i32, vp], i32),
+                    "sat_compute_dist_chained": ([vp, vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_box_filter": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i32, vp], i32),
                     "sat_comm_unique_id": ([vp], i32),
                     "sat_comm_create": ([ctypes.POINTER(vp), vp, i32, i32, i32], i32),
@@ -421,3 +424,51 @@ def dist_carry(gathered, rank: int, pair: int, plan: Plan | None = None, stream=
                                 carry.data_ptr(), _stream_ptr(stream, gathered.device)),
            "sat_dist_carry")
     return carry
+
+
+# ---------------------------------------------------------------------------
+# Chained row bands (single-pass multi-GPU path)
+
+def chain_bytes(pair: int, w: int) -> int:
+    """Bytes of one chain buffer (tagged carry vectors of a w-wide row)."""
+    return int(lib().sat_chain_bytes(pair, w))
+
+
+def new_chain_buffer(pair: int, w: int, device=None):
+    """A zero-filled, 16-byte aligned chain buffer (uint8 CUDA tensor)."""
+    torch = _torch()
+    return torch.zeros(chain_bytes(pair, w), dtype=torch.uint8, device=device or "cuda")
+
+
+def sat_band_chained(x, chain_in, chain_out, epoch: int, out=None, plan: Plan | None = None,
+                     stream=None):
+    """SAT of one band of a chain: waits (in the kernel) for the band above's
+    bottom row in chain_in, publishes its own bottom row into chain_out."""
+    torch = _torch()
+    pair = pair_of_dtype(x.dtype)
+    H, W = x.shape
+    if out is None:
+        out = torch.empty(x.shape, dtype=out_dtype(pair), device=x.device)
+    p = plan if plan is not None else _plan_for(x.device, pair, H, W, 1)
+    _check(lib().sat_compute_band_chained(
+        p.handle, x.data_ptr(), out.data_ptr(), H, W, _row_layout(x)[0], _row_layout(out)[0],
+        chain_in.data_ptr() if chain_in is not None else None,
+        chain_out.data_ptr() if chain_out is not None else None, epoch, pair,
+        _stream_ptr(stream, x.device)), "sat_compute_band_chained")
+    return out
+
+
+def sat_dist_chained(band, comm: SatComm, out=None, plan: Plan | None = None, stream=None):
+    """Row-banded SAT across ranks with chained carries over peer memory (one
+    kernel per rank, no column-sum pass)."""
+    torch = _torch()
+    pair = pair_of_dtype(band.dtype)
+    if out is None:
+        out = torch.empty(band.shape, dtype=out_dtype(pair), device=band.device)
+    H, W = band.shape
+    p = plan if plan is not None else _plan_for(band.device, pair, max(H, 1), W, 1)
+    _check(lib().sat_compute_dist_chained(p.handle, comm._h, band.data_ptr(), out.data_ptr(), H, W,
+                                          _row_layout(band)[0], _row_layout(out)[0], pair,
+                                          _stream_ptr(stream, band.device)),
+           "sat_compute_dist_chained")
+    return out

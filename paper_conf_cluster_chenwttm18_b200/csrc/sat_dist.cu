@@ -227,11 +227,33 @@ sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, 
 
 using namespace sat;
 
+// Chained-band state (sat_compute_dist_chained): this rank's receive buffer
+// for the carry vectors of the rank above, and the peer-mapped receive buffer
+// of the rank below (CUDA IPC over NVLink), exchanged once per width.
+struct ChainBufs {
+  int64_t w = 0;
+  size_t bytes = 0;
+  void* recv = nullptr;       // own, written by rank - 1
+  void* peer_recv = nullptr;  // rank + 1's, opened through its IPC handle
+  void* hdl_dev = nullptr;    // [nranks] IPC handles (allgather staging)
+  int* flag_dev = nullptr;    // [nranks] barrier words
+  uint32_t epoch = 0;
+};
+
 struct sat_comm_st {
   ncclComm_t comm = nullptr;
   int nranks = 0, rank = 0, device = 0;
   DistBufs bufs;
+  ChainBufs chain;
 };
+
+static void free_chain(ChainBufs& c) {
+  if (c.peer_recv) cudaIpcCloseMemHandle(c.peer_recv);
+  if (c.recv) cudaFree(c.recv);
+  if (c.hdl_dev) cudaFree(c.hdl_dev);
+  if (c.flag_dev) cudaFree(c.flag_dev);
+  c = ChainBufs();
+}
 
 static void free_bufs(DistBufs& b) {
   if (b.partial) cudaFree(b.partial);
@@ -298,6 +320,7 @@ sat_status sat_comm_destroy(sat_comm comm) {
   DeviceGuard g(comm->device);
   cudaDeviceSynchronize();
   free_bufs(comm->bufs);
+  free_chain(comm->chain);
   if (comm->comm) nccl().CommDestroy(comm->comm);
   delete comm;
   return SAT_OK;
@@ -371,6 +394,100 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
   return launch(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
                 band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1,
                 comm->rank > 0 ? b.carry : nullptr, s);
+}
+
+
+size_t sat_chain_bytes(sat_pair pair, int64_t w) {
+  if (w <= 0 || (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F)) return 0;
+  // one tagged 64-bit word per 32-bit half of each output element, per chunk
+  const int64_t tw = tile_w(pair);
+  return (size_t)((w + tw - 1) / tw) * (size_t)tw * out_size(pair) * 2;
+}
+
+sat_status sat_compute_band_chained(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                                    int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                                    const void* chain_in, void* chain_out, uint32_t chain_epoch,
+                                    sat_pair pair, void* stream) {
+  if (h <= 0 || w <= 0) return fail(SAT_ERR_INVALID_ARGUMENT, "a chained band needs h, w >= 1");
+  if (chain_epoch == 0 || chain_epoch >= (1u << 30))
+    return fail(SAT_ERR_INVALID_ARGUMENT, "chain_epoch must be in [1, 2^30)");
+  if (((uintptr_t)chain_in | (uintptr_t)chain_out) % 16 != 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "chain buffers must be 16-byte aligned");
+  bool empty = false;
+  sat_status st = validate(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
+                           h * in_pitch_bytes, h * out_pitch_bytes, 1, pair, &empty);
+  if (st != SAT_OK || empty) return st;
+  DeviceGuard g(plan->device);
+  const ChainSpec chain{chain_in, chain_out, chain_epoch};
+  return launch(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes, h * in_pitch_bytes,
+                h * out_pitch_bytes, 1, nullptr, static_cast<cudaStream_t>(stream), nullptr, &chain);
+}
+
+sat_status sat_compute_dist_chained(sat_plan plan, sat_comm comm, const void* in_band,
+                                    void* out_band, int64_t band_h, int64_t w,
+                                    int64_t in_pitch_bytes, int64_t out_pitch_bytes, sat_pair pair,
+                                    void* stream) {
+  if (!comm) return fail(SAT_ERR_INVALID_ARGUMENT, "comm is NULL");
+  if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (band_h <= 0 || w <= 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "every rank needs a band of >= 1 row (H >= nranks)");
+  bool empty = false;
+  sat_status st = validate(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
+                           band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1, pair, &empty);
+  if (st != SAT_OK) return st;
+  DeviceGuard g(plan->device);
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (comm->nranks == 1)
+    return launch(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
+                  band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1, nullptr, s);
+  ChainBufs& c = comm->chain;
+  const size_t bytes = sat_chain_bytes(pair, w);
+  if (c.bytes < bytes) {  // (re)build: collective, every rank calls with the same w
+    cudaStreamSynchronize(s);
+    free_chain(c);
+    cudaError_t e = cudaMalloc(&c.recv, bytes);
+    if (e == cudaSuccess) e = cudaMemset(c.recv, 0, bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&c.hdl_dev, (size_t)comm->nranks * sizeof(cudaIpcMemHandle_t));
+    if (e == cudaSuccess) e = cudaMalloc(&c.flag_dev, (size_t)comm->nranks * 2 * sizeof(int));
+    cudaIpcMemHandle_t mine;
+    if (e == cudaSuccess) e = cudaIpcGetMemHandle(&mine, c.recv);
+    if (e == cudaSuccess)
+      e = cudaMemcpy(static_cast<char*>(c.hdl_dev) + comm->rank * sizeof(mine), &mine, sizeof(mine),
+                     cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      free_chain(c);
+      return cuda_fail(e, "chain buffers");
+    }
+    ncclResult_t r = nccl().AllGather(static_cast<char*>(c.hdl_dev) + comm->rank * sizeof(mine),
+                                      c.hdl_dev, sizeof(mine), ncclUint8, comm->comm, s);
+    if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather(ipc handles)");
+    e = cudaStreamSynchronize(s);
+    if (e == cudaSuccess && comm->rank + 1 < comm->nranks) {
+      cudaIpcMemHandle_t below;
+      e = cudaMemcpy(&below, static_cast<char*>(c.hdl_dev) + (comm->rank + 1) * sizeof(below),
+                     sizeof(below), cudaMemcpyDeviceToHost);
+      if (e == cudaSuccess) e = cudaIpcOpenMemHandle(&c.peer_recv, below, cudaIpcMemLazyEnablePeerAccess);
+    }
+    if (e != cudaSuccess) {
+      free_chain(c);
+      return cuda_fail(e, "chain peer mapping");
+    }
+    c.bytes = bytes;
+    c.w = w;
+  }
+  if (++c.epoch >= (1u << 30)) {  // tags hold 30 epoch bits: clear and restart (collective)
+    cudaError_t e = cudaMemsetAsync(c.recv, 0, c.bytes, s);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(chain)");
+    c.epoch = 1;
+  }
+  // Barrier on the stream: no rank overwrites its peer's receive buffer for this
+  // call before that peer has finished reading it in the previous call.
+  ncclResult_t r = nccl().AllGather(c.flag_dev + comm->rank, c.flag_dev + comm->nranks, 1,
+                                    ncclInt32, comm->comm, s);
+  if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather(barrier)");
+  const ChainSpec chain{comm->rank > 0 ? c.recv : nullptr, c.peer_recv, c.epoch};
+  return launch(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
+                band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1, nullptr, s, nullptr, &chain);
 }
 
 }  // extern "C"

@@ -51,9 +51,16 @@ struct ExSpec {
   int64_t out_cols;
   uint64_t nval_bits;
 };
+// Chained bands: per-chunk tagged carry vectors in (from the band above) and
+// out (this band's bottom row, for the band below); see KParams.
+struct ChainSpec {
+  const void* in;
+  void* out;
+  uint32_t epoch;
+};
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
-                  cudaStream_t stream, const ExSpec* ex = nullptr);
+                  cudaStream_t stream, const ExSpec* ex = nullptr, const ChainSpec* chain = nullptr);
 void host_path_release(sat_plan_st* pl);
 
 struct DeviceGuard {

@@ -197,6 +197,13 @@ struct KParams {
   // column x + 1; column 0 holds nval; columns >= out_cols are not written.
   int64_t out_cols;
   uint64_t nval_bits;                    // nVal, a TB value's bits (added to every element)
+  // Chained bands: the carry row S(r0-1, .) arrives per
+  // chunk as an epoch-tagged vector (payload layout) written by the kernel of
+  // the band above -- possibly on another GPU through peer memory -- and this
+  // band's bottom row S(r1-1, .) is published the same way for the band below.
+  const uint64_t* chain_in;              // [nchunks][kVecWords] or NULL
+  uint64_t* chain_out;                   // [nchunks][kVecWords] or NULL
+  uint32_t chain_epoch;                  // >= 1; tag = (chain_epoch << 2) | kStIncl
 };
 
 // Optional phase profiling (debug builds with -DSAT_PROFILE): per-CTA shared
@@ -855,6 +862,58 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
   }
 }
 
+// Chained-band carry vectors: system-scope relaxed 64-bit accesses (peer GPU
+// memory over NVLink keeps aligned 8-byte stores single-copy atomic, so a word
+// with the expected tag also holds its value).
+__device__ __forceinline__ void st_sys_v2_u64(uint64_t* q, uint64_t a, uint64_t b) {
+  asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(q), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ void ld_sys_v2_u64(const uint64_t* q, uint64_t& a, uint64_t& b) {
+  asm volatile("ld.relaxed.sys.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(q) : "memory");
+}
+
+template <int P>
+__device__ __forceinline__ void chain_publish(const KParams& p, int32_t chunk,
+                                              const typename Cfg<P>::TB (&v)[Cfg<P>::G][Cfg<P>::E],
+                                              int lane) {
+  using C = Cfg<P>;
+  uint64_t* row = p.chain_out + (int64_t)chunk * kVecWords<P>;
+#pragma unroll
+  for (int g = 0; g < C::G; ++g) {
+    uint64_t w[4];
+    Tag<kBase<P>>::enc(v[g], (p.chain_epoch << 2) | kStIncl, w);
+    uint64_t* dst = row + (g * 32 + lane) * 4;
+    st_sys_v2_u64(dst, w[0], w[1]);
+    st_sys_v2_u64(dst + 2, w[2], w[3]);
+  }
+}
+
+template <int P>
+__device__ __forceinline__ void chain_wait(const KParams& p, int32_t chunk,
+                                           typename Cfg<P>::TB (&V)[Cfg<P>::G][Cfg<P>::E], int lane) {
+  using C = Cfg<P>;
+  const uint64_t* row = p.chain_in + (int64_t)chunk * kVecWords<P>;
+  const uint32_t want = (p.chain_epoch << 2) | kStIncl;
+  for (;;) {
+    bool ok = true;
+    uint64_t w[C::G][4];
+#pragma unroll
+    for (int g = 0; g < C::G; ++g) {
+      const uint64_t* src = row + (g * 32 + lane) * 4;
+      ld_sys_v2_u64(src, w[g][0], w[g][1]);
+      ld_sys_v2_u64(src + 2, w[g][2], w[g][3]);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) ok &= (uint32_t)(w[g][e] >> 32) == want;
+    }
+    if (__all_sync(kFull, ok)) {
+#pragma unroll
+      for (int g = 0; g < C::G; ++g) Tag<kBase<P>>::dec(w[g], V[g]);
+      return;
+    }
+    __nanosleep(64);
+  }
+}
+
 template <int P>
 __device__ __forceinline__ void load_carry_in(const KParams& p, int32_t chunk,
                                               typename Cfg<P>::TB (&V)[Cfg<P>::G][Cfg<P>::E],
@@ -923,7 +982,10 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
   const bool has_succ = tail_last_k + 1 < bpi;
   const bool head_self = (k0 == 0);
   TB carry0[C::G][C::E];
-  load_carry_in<P>(p, chunk, carry0, lane);
+  if (p.chain_in != nullptr && (head_self || tail_self))
+    chain_wait<P>(p, chunk, carry0, lane);  // the band above publishes it chunk by chunk
+  else
+    load_carry_in<P>(p, chunk, carry0, lane);
   if (has_succ) {
     if (tail_self) {
       TB incl[C::G][C::E];
@@ -989,6 +1051,8 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
       }
       if (++k == bpi) k = 0;
     }
+    // The image's bottom row S(r1-1, .) = the tail segment's inclusive value.
+    if (!has_succ && p.chain_out != nullptr) chain_publish<P>(p, chunk, run, lane);
   }
   if (has_succ && !tail_self) {
     TB incl[C::G][C::E];

@@ -69,7 +69,8 @@ static EncodeTiledFn get_encode() {
 template <int P>
 static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
                            int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
-                           const void* carry_in, cudaStream_t stream, const ExSpec* ex) {
+                           const void* carry_in, cudaStream_t stream, const ExSpec* ex,
+                           const ChainSpec* chain) {
   using C = Cfg<P>;
   const bool tma = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
                    getenv_int("SAT_FORCE_GENERIC", 0) == 0;
@@ -89,6 +90,9 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.carry_in = carry_in;
   kp.out_cols = ex ? ex->out_cols : w;
   kp.nval_bits = ex ? ex->nval_bits : 0;
+  kp.chain_in = chain ? static_cast<const uint64_t*>(chain->in) : nullptr;
+  kp.chain_out = chain ? static_cast<uint64_t*>(chain->out) : nullptr;
+  kp.chain_epoch = chain ? chain->epoch : 0;
   if ((kp.total_bands + (P >= kShort ? 1 : 0)) / (P >= kShort ? 2 : 1) * kp.nchunks > pl->max_tiles)
     return fail(SAT_ERR_INVALID_ARGUMENT, "problem needs %lld tiles, plan holds %lld",
                 (long long)(kp.total_bands * kp.nchunks), (long long)pl->max_tiles);
@@ -241,7 +245,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
 
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
-                  cudaStream_t stream, const ExSpec* ex) {
+                  cudaStream_t stream, const ExSpec* ex, const ChainSpec* chain) {
   // Short, wide images: 32-row bands give only H/4 compute warps in total
   // (2 CTAs of 8 warps per SM leave most SMs idle below ~140 bands); 16-row
   // bands (2 rows per warp) double the warps in flight.
@@ -256,20 +260,20 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
   if (use_short) {
     switch (pl->pair) {
       case SAT_8U_32S:
-        return launch_t<P8U32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+        return launch_t<P8U32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
       case SAT_32F_32F:
-        return launch_t<P32F32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+        return launch_t<P32F32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
       case SAT_64F_64F:
-        return launch_t<P64F64F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+        return launch_t<P64F64F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
     }
   }
   switch (pl->pair) {
     case SAT_8U_32S:
-      return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+      return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
     case SAT_32F_32F:
-      return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+      return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
     case SAT_64F_64F:
-      return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex);
+      return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
