@@ -110,3 +110,33 @@ def test_chained_invalid_arguments():
                                       None, b.data_ptr() + 8, 1, 0, None) == 1  # alignment
     assert sat.chain_bytes(0, 257) == 2 * 256 * 4 * 2
     p.close()
+
+
+@pytest.mark.parametrize("d", [np.uint8, np.float32])
+def test_chained_bands_concurrent_streams(monkeypatch, d):
+    """The bands run CONCURRENTLY on separate streams (as peers do on separate
+    GPUs): each kernel's persistent grid is capped (SAT_MAX_CLUSTERS) so that
+    all bands are co-resident whatever order the hardware starts them in, and
+    the lower bands' top clusters really wait inside the kernel for chunks
+    still being produced above them."""
+    torch, sat = _t(), _sat()
+    P = 3
+    monkeypatch.setenv("SAT_MAX_CLUSTERS", "16")  # 3 x 16 clusters x 4 CTAs <= 2 CTAs/SM x 148
+    monkeypatch.setenv("SAT_SHORT", "0")
+    H, W = 3 * 2048, 8192
+    x = torch.empty((H, W), dtype=_tdt(d), device="cuda")
+    satgen.fill_device(x, seed=91)
+    pair = sat.pair_of_dtype(x.dtype)
+    bufs = [sat.new_chain_buffer(pair, W) for _ in range(P - 1)]
+    out = torch.empty((H, W), dtype=sat.out_dtype(pair), device="cuda")
+    plans = [sat.Plan(pair, H, W, 1) for _ in range(P)]
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    torch.cuda.synchronize()
+    for r in reversed(range(P)):  # lowest band first: it must wait for the others
+        r0, r1 = sat.band_partition(H, P, r)
+        with torch.cuda.stream(streams[r]):
+            sat.sat_band_chained(x[r0:r1], bufs[r - 1] if r > 0 else None,
+                                 bufs[r] if r < P - 1 else None, 1, out=out[r0:r1],
+                                 plan=plans[r], stream=streams[r])
+    torch.cuda.synchronize()
+    _check(out.cpu().numpy(), oracle.sat(x.cpu().numpy()), d, "concurrent chain")
