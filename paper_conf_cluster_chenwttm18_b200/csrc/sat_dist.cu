@@ -7,7 +7,7 @@
 //                              in u32 for 8u, compensated fp64 for 32f/64f);
 //   2. ncclAllGather         : every rank receives all ranks' W-vectors over
 //                              NVLink/NVSwitch (the one data exchange);
-//   3. sat_band_carry_kernel : exclusive prefix over lower ranks, then the
+//   3. sat_carry_*_kernels   : exclusive prefix over lower ranks, then the
 //                              horizontal inclusive prefix over x, rounded
 //                              once to T_B -> the carry-in row;
 //   4. sat_tile_kernel       : the band's SAT with that carry-in on its top
@@ -88,6 +88,43 @@ __global__ void sat_colsum_kernel(const char* __restrict__ in, int64_t h, int64_
   partial[(int64_t)blockIdx.y * w + x] = s + comp;
 }
 
+// Vectorised variant: each thread sums V adjacent columns with one 4/16-byte
+// load per row (the scalar kernel issues 4-byte loads; this halves the pass).
+template <typename TA, typename ACC, int V>
+__global__ void sat_colsum_vec_kernel(const char* __restrict__ in, int64_t h, int64_t w,
+                                      int64_t pitch, int64_t rows_per_split, ACC* __restrict__ partial) {
+  const int64_t x = ((int64_t)blockIdx.x * kColsumThreads + threadIdx.x) * V;
+  const int64_t y0 = (int64_t)blockIdx.y * rows_per_split;
+  const int64_t y1 = min(h, y0 + rows_per_split);
+  if (x >= w) return;
+  ACC s[V], comp[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) s[v] = comp[v] = ACC(0);
+  for (int64_t y = y0; y < y1; ++y) {
+    TA a[V];
+    const TA* src = reinterpret_cast<const TA*>(in + y * pitch) + x;
+    if constexpr (sizeof(TA) * V == 16) {
+      *reinterpret_cast<uint4*>(a) = __ldg(reinterpret_cast<const uint4*>(src));
+    } else {
+      static_assert(sizeof(TA) * V == 4, "4- or 16-byte vectors");
+      *reinterpret_cast<uint32_t*>(a) = __ldg(reinterpret_cast<const uint32_t*>(src));
+    }
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const ACC val = (ACC)a[v];
+      if constexpr (sizeof(ACC) == 8) {
+        const ACC t = s[v] + val;
+        comp[v] += (fabs(s[v]) >= fabs(val)) ? ((s[v] - t) + val) : ((val - t) + s[v]);
+        s[v] = t;
+      } else {
+        s[v] += val;
+      }
+    }
+  }
+#pragma unroll
+  for (int v = 0; v < V; ++v) partial[(int64_t)blockIdx.y * w + x + v] = s[v] + comp[v];
+}
+
 template <typename ACC>
 __global__ void sat_colsum_reduce_kernel(const ACC* __restrict__ partial, int splits, int64_t w,
                                          ACC* __restrict__ out) {
@@ -107,61 +144,81 @@ __global__ void sat_colsum_reduce_kernel(const ACC* __restrict__ partial, int sp
   out[x] = s + comp;
 }
 
-// One CTA: c(x) = sum_{r' < rank} gathered[r'][x]; carry(x) = sum_{x' <= x} c(x').
-constexpr int kCarryThreads = 1024;
+// Carry row, three coalesced phases (was one CTA walking strided segments):
+//   c(x) = sum_{r' < rank} gathered[r'][x],   carry(x) = sum_{x' <= x} c(x').
+// Phase 1: each CTA scans kCarryItems * kCarryThreads consecutive x (thread-
+// serial over kCarryItems, then warp shuffles and a shared-memory pass over
+// the warps) and writes local prefixes + its total; phase 2 (one thread):
+// compensated exclusive scan of the CTA totals; phase 3: add and round once
+// to T_B.
+constexpr int kCarryThreads = 1024, kCarryItems = 4;
+constexpr int kCarryTile = kCarryThreads * kCarryItems;
 
-template <typename ACC, typename TB>
+template <typename ACC>
+__device__ __forceinline__ ACC warp_incl_scan(ACC v, int lane) {
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const ACC o = __shfl_up_sync(0xffffffffu, v, d);
+    if (lane >= d) v += o;
+  }
+  return v;
+}
+
+template <typename ACC>
 __global__ void __launch_bounds__(kCarryThreads)
-    sat_band_carry_kernel(const ACC* __restrict__ gathered, int rank, int64_t w, TB* __restrict__ carry) {
-  __shared__ ACC part[kCarryThreads];
-  const int64_t seg = (w + kCarryThreads - 1) / kCarryThreads;
-  const int64_t x0 = (int64_t)threadIdx.x * seg;
-  const int64_t x1 = min(w, x0 + seg);
-  // pass 1: segment total of c(x)
-  ACC tot = ACC(0), totc = ACC(0);
-  for (int64_t x = x0; x < x1; ++x) {
+    sat_carry_scan_kernel(const ACC* __restrict__ gathered, int rank, int64_t w,
+                          ACC* __restrict__ local, ACC* __restrict__ tile_tot) {
+  __shared__ ACC wsum[kCarryThreads / 32];
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int64_t base = (int64_t)blockIdx.x * kCarryTile + (int64_t)tid * kCarryItems;
+  ACC v[kCarryItems];
+  ACC run = ACC(0);
+#pragma unroll
+  for (int k = 0; k < kCarryItems; ++k) {
+    const int64_t x = base + k;
     ACC c = ACC(0);
-    for (int r = 0; r < rank; ++r) c += gathered[(int64_t)r * w + x];
-    if constexpr (sizeof(ACC) == 8) {
-      const ACC t = tot + c;
-      totc += (fabs(tot) >= fabs(c)) ? ((tot - t) + c) : ((c - t) + tot);
-      tot = t;
-    } else {
-      tot += c;
-    }
+    if (x < w)
+      for (int r = 0; r < rank; ++r) c += gathered[(int64_t)r * w + x];
+    run += c;
+    v[k] = run;
   }
-  part[threadIdx.x] = tot + totc;
+  const ACC incl = warp_incl_scan(run, lane);
+  if (lane == 31) wsum[wid] = incl;
   __syncthreads();
-  // exclusive scan of segment totals (serial by thread 0: 1024 adds)
-  if (threadIdx.x == 0) {
-    ACC run = ACC(0), runc = ACC(0);
-    for (int i = 0; i < kCarryThreads; ++i) {
-      const ACC v = part[i];
-      part[i] = run + runc;
-      if constexpr (sizeof(ACC) == 8) {
-        const ACC t = run + v;
-        runc += (fabs(run) >= fabs(v)) ? ((run - t) + v) : ((v - t) + run);
-        run = t;
-      } else {
-        run += v;
-      }
-    }
+  if (wid == 0) {
+    const ACC ws = warp_incl_scan(wsum[lane], lane);
+    wsum[lane] = ws;
   }
   __syncthreads();
-  // pass 2: inclusive prefix within the segment, rounded once to T_B
-  ACC run = part[threadIdx.x], runc = ACC(0);
-  for (int64_t x = x0; x < x1; ++x) {
-    ACC c = ACC(0);
-    for (int r = 0; r < rank; ++r) c += gathered[(int64_t)r * w + x];
+  const ACC off = (incl - run) + (wid > 0 ? wsum[wid - 1] : ACC(0));
+#pragma unroll
+  for (int k = 0; k < kCarryItems; ++k)
+    if (base + k < w) local[base + k] = off + v[k];
+  if (tid == kCarryThreads - 1) tile_tot[blockIdx.x] = wsum[kCarryThreads / 32 - 1];
+}
+
+template <typename ACC>
+__global__ void sat_carry_offsets_kernel(ACC* __restrict__ tile_tot, int64_t ntiles) {
+  if (threadIdx.x != 0) return;
+  ACC run = ACC(0), runc = ACC(0);
+  for (int64_t i = 0; i < ntiles; ++i) {
+    const ACC v = tile_tot[i];
+    tile_tot[i] = run + runc;  // exclusive
     if constexpr (sizeof(ACC) == 8) {
-      const ACC t = run + c;
-      runc += (fabs(run) >= fabs(c)) ? ((run - t) + c) : ((c - t) + run);
+      const ACC t = run + v;
+      runc += (fabs(run) >= fabs(v)) ? ((run - t) + v) : ((v - t) + run);
       run = t;
     } else {
-      run += c;
+      run += v;
     }
-    carry[x] = (TB)(run + runc);
   }
+}
+
+template <typename ACC, typename TB>
+__global__ void sat_carry_finish_kernel(const ACC* __restrict__ local, const ACC* __restrict__ tile_off,
+                                        int64_t w, TB* __restrict__ carry) {
+  const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (x < w) carry[x] = (TB)(tile_off[x / kCarryTile] + local[x]);
 }
 
 size_t acc_size(sat_pair p) { return p == SAT_8U_32S ? 4 : 8; }
@@ -188,6 +245,27 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
   const int used = (int)((h + rps - 1) / rps);
   dim3 grid((unsigned)((w + kColsumThreads - 1) / kColsumThreads), (unsigned)used);
   const char* p = static_cast<const char*>(in);
+  const int vw = pair == SAT_64F_64F ? 2 : 4;  // elements per vector load
+  const int vb = pair == SAT_8U_32S ? 4 : 16;  // bytes per vector load
+  if (w % vw == 0 && pitch % vb == 0 && (uintptr_t)in % vb == 0) {
+    dim3 gv((unsigned)((w / vw + kColsumThreads - 1) / kColsumThreads), (unsigned)used);
+    switch (pair) {
+      case SAT_8U_32S:
+        sat_colsum_vec_kernel<uint8_t, uint32_t, 4><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (uint32_t*)partial);
+        sat_colsum_reduce_kernel<uint32_t><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((uint32_t*)partial, used, w, (uint32_t*)out);
+        break;
+      case SAT_32F_32F:
+        sat_colsum_vec_kernel<float, double, 4><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
+        sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
+        break;
+      case SAT_64F_64F:
+        sat_colsum_vec_kernel<double, double, 2><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
+        sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
+        break;
+    }
+    cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? SAT_OK : cuda_fail(e, "sat_colsum_vec_kernel launch");
+  }
   switch (pair) {
     case SAT_8U_32S:
       sat_colsum_kernel<uint8_t, uint32_t><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (uint32_t*)partial);
@@ -208,19 +286,37 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
 
 sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, void* carry,
                       cudaStream_t s) {
+  // scratch: local prefixes [w] + tile totals (stream-ordered allocation)
+  const int64_t ntiles = (w + kCarryTile - 1) / kCarryTile;
+  void* scratch = nullptr;
+  cudaError_t e = cudaMallocAsync(&scratch, (size_t)(w + ntiles) * 8, s);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMallocAsync(carry scratch)");
+  const unsigned fin = (unsigned)((w + 255) / 256);
   switch (pair) {
-    case SAT_8U_32S:
-      sat_band_carry_kernel<uint32_t, uint32_t><<<1, kCarryThreads, 0, s>>>((const uint32_t*)gathered, rank, w, (uint32_t*)carry);
+    case SAT_8U_32S: {
+      uint32_t* loc = (uint32_t*)scratch;
+      uint32_t* tt = loc + w;
+      sat_carry_scan_kernel<uint32_t><<<(unsigned)ntiles, kCarryThreads, 0, s>>>((const uint32_t*)gathered, rank, w, loc, tt);
+      sat_carry_offsets_kernel<uint32_t><<<1, 32, 0, s>>>(tt, ntiles);
+      sat_carry_finish_kernel<uint32_t, uint32_t><<<fin, 256, 0, s>>>(loc, tt, w, (uint32_t*)carry);
       break;
+    }
     case SAT_32F_32F:
-      sat_band_carry_kernel<double, float><<<1, kCarryThreads, 0, s>>>((const double*)gathered, rank, w, (float*)carry);
+    case SAT_64F_64F: {
+      double* loc = (double*)scratch;
+      double* tt = loc + w;
+      sat_carry_scan_kernel<double><<<(unsigned)ntiles, kCarryThreads, 0, s>>>((const double*)gathered, rank, w, loc, tt);
+      sat_carry_offsets_kernel<double><<<1, 32, 0, s>>>(tt, ntiles);
+      if (pair == SAT_32F_32F)
+        sat_carry_finish_kernel<double, float><<<fin, 256, 0, s>>>(loc, tt, w, (float*)carry);
+      else
+        sat_carry_finish_kernel<double, double><<<fin, 256, 0, s>>>(loc, tt, w, (double*)carry);
       break;
-    case SAT_64F_64F:
-      sat_band_carry_kernel<double, double><<<1, kCarryThreads, 0, s>>>((const double*)gathered, rank, w, (double*)carry);
-      break;
+    }
   }
-  cudaError_t e = cudaGetLastError();
-  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "sat_band_carry_kernel launch");
+  e = cudaGetLastError();
+  cudaFreeAsync(scratch, s);
+  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "carry kernels launch");
 }
 
 }  // namespace sat
