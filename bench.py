@@ -447,8 +447,10 @@ def run_banded(args, rank, world, local_rank, H=65536, W=65536, pair=1, seed=100
     del band, out
     torch.cuda.empty_cache()
     px = H * W
-    # per rank: the band is read twice (column sums, then the SAT) and written once
-    per_rank_bytes = (r1 - r0) * W * (2 * IN_B[pair] + OUT_B[pair])
+    # per rank: the band is read twice (column sums, then the SAT) and written
+    # once; a single rank has no carry to exchange (sat_compute_dist runs the SAT only)
+    reads = 2 if world > 1 else 1
+    per_rank_bytes = (r1 - r0) * W * (reads * IN_B[pair] + OUT_B[pair])
     return {"workload": "huge-65536sq-32f32f row-banded", "n_gpus": world, "steps": steps,
             "ms_per_step": ms, "value": px / (ms * 1e-3) / 1e9, "unit": "Gpx/s",
             "scaling": "strong", "parallelism": f"row bands x{world} (ncclAllGather carry)",
