@@ -203,3 +203,12 @@ def box_filter(A: np.ndarray, ry: int, rx: int) -> np.ndarray:
     if pair == PAIR_8U32S:
         return (out & 0xFFFFFFFF).astype(np.uint32).view(np.int32)
     return out
+
+
+def sat_8u32f(A: np.ndarray) -> np.ndarray:
+    """Reference for the 8u->32f pair (NPP's nppiIntegral_8u32f):
+    the EXACT inclusive sums of the uint8 image, as fp64 (the double-double
+    recurrence of `sat` is exact for integer sums below 2^53); the GPU's fp32
+    result is judged against it with the 32f bar (1e-4 relative)."""
+    assert A.dtype == np.uint8
+    return sat(np.ascontiguousarray(A, dtype=np.float64))

@@ -79,3 +79,15 @@ def test_exclusive_empty_shapes():
     J = oracle.sat_exclusive(A, full=True, nval=4)
     assert J.shape == (1, 6) and np.all(J == 4)
     assert oracle.sat_exclusive(A, full=False).shape == (0, 5)
+
+
+def test_8u32f_reference_is_exact_sum():
+    """oracle.sat_8u32f equals the brute-force integer rectangle sums (tiny)
+    and the exact int64 cumsums past 2^32 (where 8u->32s wraps)."""
+    A = RNG.integers(0, 256, (6, 9)).astype(np.uint8)
+    ref = np.array([[int(A[:i + 1, :j + 1].astype(np.int64).sum()) for j in range(9)] for i in range(6)],
+                   dtype=np.float64)
+    assert np.array_equal(oracle.sat_8u32f(A), ref)
+    B = np.full((300, 70000), 255, dtype=np.uint8)  # total 5.4e9 > 2^32
+    got = oracle.sat_8u32f(B)
+    assert got[-1, -1] == 255.0 * 300 * 70000
