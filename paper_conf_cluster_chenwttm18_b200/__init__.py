@@ -17,9 +17,9 @@ import os
 import threading
 
 __all__ = ["SatError", "Plan", "sat", "sat_host", "SatComm", "sat_dist", "band_partition",
-           "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "lib", "LIB_PATH"]
+           "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "PAIR_8U_32F", "lib", "LIB_PATH"]
 
-PAIR_8U_32S, PAIR_32F_32F, PAIR_64F_64F = 0, 1, 2
+PAIR_8U_32S, PAIR_32F_32F, PAIR_64F_64F, PAIR_8U_32F = 0, 1, 2, 3
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("SAT_LIBRARY") or os.path.join(_HERE, "libsat.so")
 COMM_ID_BYTES = 128
@@ -91,17 +91,24 @@ def _torch():
     return torch
 
 
-def pair_of_dtype(dtype) -> int:
+def pair_of_dtype(dtype, out=None) -> int:
+    """Type pair of an input dtype; uint8 with a float32 output is 8u->32f."""
     torch = _torch()
     m = {torch.uint8: PAIR_8U_32S, torch.float32: PAIR_32F_32F, torch.float64: PAIR_64F_64F}
     if dtype not in m:
         raise TypeError(f"unsupported input dtype {dtype}; expected uint8, float32 or float64")
+    if dtype == torch.uint8 and out == torch.float32:
+        return PAIR_8U_32F
     return m[dtype]
 
 
 def out_dtype(pair: int):
     torch = _torch()
-    return {PAIR_8U_32S: torch.int32, PAIR_32F_32F: torch.float32, PAIR_64F_64F: torch.float64}[pair]
+    return {PAIR_8U_32S: torch.int32, PAIR_32F_32F: torch.float32, PAIR_64F_64F: torch.float64,
+            PAIR_8U_32F: torch.float32}[pair]
+
+
+_out_dtype_of = out_dtype  # for functions whose `out_dtype` parameter shadows the helper
 
 
 def _stream_ptr(stream, device):
@@ -199,17 +206,18 @@ def _row_layout(t):
     return pitch, img
 
 
-def sat(x, out=None, plan: Plan | None = None, stream=None):
+def sat(x, out=None, plan: Plan | None = None, stream=None, out_dtype=None):
     """Inclusive SAT of a CUDA tensor [H, W] or [N, H, W] (uint8/float32/float64).
 
-    Returns ``out`` (allocated if None: int32 / float32 / float64)."""
+    Returns ``out`` (allocated if None: int32 / float32 / float64).  A uint8
+    input with out_dtype (or out) float32 selects the 8u->32f pair."""
     torch = _torch()
     if not x.is_cuda:
         raise ValueError("sat() needs a CUDA tensor (use sat_host for host arrays)")
-    pair = pair_of_dtype(x.dtype)
+    pair = pair_of_dtype(x.dtype, out.dtype if out is not None else out_dtype)
     if out is None:
-        out = torch.empty(x.shape, dtype=out_dtype(pair), device=x.device)
-    elif out.dtype != out_dtype(pair) or out.shape != x.shape or out.device != x.device:
+        out = torch.empty(x.shape, dtype=_out_dtype_of(pair), device=x.device)
+    elif out.dtype != _out_dtype_of(pair) or out.shape != x.shape or out.device != x.device:
         raise ValueError("out has the wrong dtype/shape/device")
     H, W = x.shape[-2], x.shape[-1]
     N = x.shape[0] if x.dim() == 3 else 1
@@ -225,26 +233,27 @@ def sat(x, out=None, plan: Plan | None = None, stream=None):
     return out
 
 
-def sat_exclusive(x, full: bool = True, nval=0, out=None, plan: Plan | None = None, stream=None):
+def sat_exclusive(x, full: bool = True, nval=0, out=None, plan: Plan | None = None, stream=None,
+                  out_dtype=None):
     """Exclusive SAT (Eq. 2) of a CUDA tensor [H, W] plus nVal on every
     element: full=True gives NPP's / OpenCV's (H+1) x (W+1) layout, full=False
     Eq. 2's H x W.  sat_compute_exclusive does all the work."""
     torch = _torch()
     if not x.is_cuda or x.dim() != 2:
         raise ValueError("sat_exclusive() needs a 2-D CUDA tensor")
-    pair = pair_of_dtype(x.dtype)
+    pair = pair_of_dtype(x.dtype, out.dtype if out is not None else out_dtype)
     H, W = x.shape
     shape = (H + 1, W + 1) if full else (H, W)
     if out is None:
         # rows padded to 16 bytes (a view), so the kernel's shifted stores stay vectorised
-        per16 = 16 // torch.empty((), dtype=out_dtype(pair)).element_size()
+        per16 = 16 // torch.empty((), dtype=_out_dtype_of(pair)).element_size()
         cols = -(-max(shape[1], 1) // per16) * per16
-        out = torch.empty((shape[0], cols), dtype=out_dtype(pair), device=x.device)[:, :shape[1]]
-    elif out.dtype != out_dtype(pair) or tuple(out.shape) != shape or out.device != x.device:
+        out = torch.empty((shape[0], cols), dtype=_out_dtype_of(pair), device=x.device)[:, :shape[1]]
+    elif out.dtype != _out_dtype_of(pair) or tuple(out.shape) != shape or out.device != x.device:
         raise ValueError("out has the wrong dtype/shape/device")
     if out.numel() == 0:
         return out
-    ctype = {0: ctypes.c_int32, 1: ctypes.c_float, 2: ctypes.c_double}[pair]
+    ctype = {0: ctypes.c_int32, 1: ctypes.c_float, 2: ctypes.c_double, 3: ctypes.c_float}[pair]
     nv = ctype(nval)
     ip = _row_layout(x)[0] if H > 0 and W > 0 else max(W, 1) * x.element_size()
     op = _row_layout(out)[0]
@@ -293,12 +302,12 @@ def box_filter(S, ry: int, rx: int, out=None, plan: Plan | None = None, stream=N
     return out
 
 
-def sat_band(x, carry_in=None, out=None, plan: Plan | None = None, stream=None):
+def sat_band(x, carry_in=None, out=None, plan: Plan | None = None, stream=None, out_dtype=None):
     """SAT of a row band given the SAT row above it (carry_in: [W] of the output dtype)."""
     torch = _torch()
-    pair = pair_of_dtype(x.dtype)
+    pair = pair_of_dtype(x.dtype, out.dtype if out is not None else out_dtype)
     if out is None:
-        out = torch.empty(x.shape, dtype=out_dtype(pair), device=x.device)
+        out = torch.empty(x.shape, dtype=_out_dtype_of(pair), device=x.device)
     H, W = x.shape
     if H == 0 or W == 0:
         return out
@@ -306,7 +315,7 @@ def sat_band(x, carry_in=None, out=None, plan: Plan | None = None, stream=None):
     op, _ = _row_layout(out)
     cptr = None
     if carry_in is not None:
-        if carry_in.dtype != out_dtype(pair) or carry_in.numel() < W or not carry_in.is_contiguous():
+        if carry_in.dtype != _out_dtype_of(pair) or carry_in.numel() < W or not carry_in.is_contiguous():
             raise ValueError("carry_in must be a contiguous [W] tensor of the output dtype")
         cptr = carry_in.data_ptr()
     p = plan if plan is not None else _plan_for(x.device, pair, H, W, 1)
@@ -322,7 +331,7 @@ def sat_host(x, out=None, plan: Plan | None = None, device=None, stream=None):
     torch = _torch()
     if x.is_cuda:
         raise ValueError("sat_host() takes a host tensor")
-    pair = pair_of_dtype(x.dtype)
+    pair = pair_of_dtype(x.dtype, out.dtype if out is not None else None)
     if out is None:
         out = torch.empty(x.shape, dtype=out_dtype(pair), pin_memory=x.is_pinned())
     dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
@@ -388,7 +397,7 @@ class SatComm:
 def sat_dist(band, comm: SatComm, out=None, plan: Plan | None = None, stream=None):
     """Row-banded SAT: `band` holds this rank's rows of one image (ranks in order)."""
     torch = _torch()
-    pair = pair_of_dtype(band.dtype)
+    pair = pair_of_dtype(band.dtype, out.dtype if out is not None else None)
     if out is None:
         out = torch.empty(band.shape, dtype=out_dtype(pair), device=band.device)
     H, W = band.shape
@@ -401,10 +410,10 @@ def sat_dist(band, comm: SatComm, out=None, plan: Plan | None = None, stream=Non
     return out
 
 
-def dist_colsum(band, plan: Plan | None = None, stream=None):
+def dist_colsum(band, plan: Plan | None = None, stream=None, pair=None):
     """Step 1 of sat_dist: the band's column totals (uint32 or float64 [W])."""
     torch = _torch()
-    pair = pair_of_dtype(band.dtype)
+    pair = pair_of_dtype(band.dtype) if pair is None else pair
     H, W = band.shape
     acc = torch.empty(W, dtype=torch.int32 if pair == PAIR_8U_32S else torch.float64, device=band.device)
     ip = band.stride(0) * band.element_size() if H > 1 else W * band.element_size()
@@ -445,7 +454,7 @@ def sat_band_chained(x, chain_in, chain_out, epoch: int, out=None, plan: Plan | 
     """SAT of one band of a chain: waits (in the kernel) for the band above's
     bottom row in chain_in, publishes its own bottom row into chain_out."""
     torch = _torch()
-    pair = pair_of_dtype(x.dtype)
+    pair = pair_of_dtype(x.dtype, out.dtype if out is not None else None)
     H, W = x.shape
     if out is None:
         out = torch.empty(x.shape, dtype=out_dtype(pair), device=x.device)
@@ -462,7 +471,7 @@ def sat_dist_chained(band, comm: SatComm, out=None, plan: Plan | None = None, st
     """Row-banded SAT across ranks with chained carries over peer memory (one
     kernel per rank, no column-sum pass)."""
     torch = _torch()
-    pair = pair_of_dtype(band.dtype)
+    pair = pair_of_dtype(band.dtype, out.dtype if out is not None else None)
     if out is None:
         out = torch.empty(band.shape, dtype=out_dtype(pair), device=band.device)
     H, W = band.shape

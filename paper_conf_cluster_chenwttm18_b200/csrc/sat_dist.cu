@@ -246,7 +246,7 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
   dim3 grid((unsigned)((w + kColsumThreads - 1) / kColsumThreads), (unsigned)used);
   const char* p = static_cast<const char*>(in);
   const int vw = pair == SAT_64F_64F ? 2 : 4;  // elements per vector load
-  const int vb = pair == SAT_8U_32S ? 4 : 16;  // bytes per vector load
+  const int vb = (pair == SAT_8U_32S || pair == SAT_8U_32F) ? 4 : 16;  // bytes per vector load
   if (w % vw == 0 && pitch % vb == 0 && (uintptr_t)in % vb == 0) {
     dim3 gv((unsigned)((w / vw + kColsumThreads - 1) / kColsumThreads), (unsigned)used);
     switch (pair) {
@@ -256,6 +256,10 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
         break;
       case SAT_32F_32F:
         sat_colsum_vec_kernel<float, double, 4><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
+        sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
+        break;
+      case SAT_8U_32F:
+        sat_colsum_vec_kernel<uint8_t, double, 4><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
         sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
         break;
       case SAT_64F_64F:
@@ -273,6 +277,10 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
       break;
     case SAT_32F_32F:
       sat_colsum_kernel<float, double><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
+      sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
+      break;
+    case SAT_8U_32F:
+      sat_colsum_kernel<uint8_t, double><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
       sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
       break;
     case SAT_64F_64F:
@@ -302,12 +310,13 @@ sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, 
       break;
     }
     case SAT_32F_32F:
+    case SAT_8U_32F:
     case SAT_64F_64F: {
       double* loc = (double*)scratch;
       double* tt = loc + w;
       sat_carry_scan_kernel<double><<<(unsigned)ntiles, kCarryThreads, 0, s>>>((const double*)gathered, rank, w, loc, tt);
       sat_carry_offsets_kernel<double><<<1, 32, 0, s>>>(tt, ntiles);
-      if (pair == SAT_32F_32F)
+      if (pair != SAT_64F_64F)
         sat_carry_finish_kernel<double, float><<<fin, 256, 0, s>>>(loc, tt, w, (float*)carry);
       else
         sat_carry_finish_kernel<double, double><<<fin, 256, 0, s>>>(loc, tt, w, (double*)carry);
@@ -494,7 +503,9 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
 
 
 size_t sat_chain_bytes(sat_pair pair, int64_t w) {
-  if (w <= 0 || (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F)) return 0;
+  if (w <= 0 || (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F &&
+                 pair != SAT_8U_32F))
+    return 0;
   // one tagged 64-bit word per 32-bit half of each output element, per chunk
   const int64_t tw = tile_w(pair);
   return (size_t)((w + tw - 1) / tw) * (size_t)tw * out_size(pair) * 2;

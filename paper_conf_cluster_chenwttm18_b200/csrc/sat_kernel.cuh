@@ -57,11 +57,11 @@
 
 namespace sat {
 
-enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2 };
+enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2, P8U32F = 3 };
 // Short-band variants (P + kShort): the same pair with 16-row bands (2 rows per
 // compute warp), chosen for short, wide images whose 32-row bands would leave
 // most of the machine idle (H / 4 compute warps in total otherwise).
-constexpr int kShort = 3;
+constexpr int kShort = 4;
 template <int P>
 constexpr int kBase = P % kShort;
 
@@ -124,6 +124,13 @@ struct Cfg<P64F64F> {
   static constexpr int NCW = 8;
   static constexpr int NSTAGE = 3;
 };
+// 8u -> 32f (NPP's nppiIntegral_8u32f): bytes in, the fp32 scans of 32f.
+template <>
+struct Cfg<P8U32F> : Cfg<P32F32F> {
+  using TA = uint8_t;
+  static constexpr int NSTAGE = 4;
+};
+
 template <int P>
 struct CfgShort : Cfg<P> {
   static constexpr int TH = Cfg<P>::TH / 2;
@@ -134,6 +141,8 @@ template <>
 struct Cfg<P32F32F + kShort> : CfgShort<P32F32F> {};
 template <>
 struct Cfg<P64F64F + kShort> : CfgShort<P64F64F> {};
+template <>
+struct Cfg<P8U32F + kShort> : CfgShort<P8U32F> {};
 
 
 // Warp roles: NCW compute warps, then the producer, then kNLB look-back warps.
@@ -176,6 +185,7 @@ constexpr int kTmemColsPerSlot = kTmemColsPerWarp<P> * (kNCW<P> / 4);  // NCW/4 
 static_assert(kTmemColsPerSlot<P8U32S> * kNTot<P8U32S> <= kTmemCols<P8U32S>, "TMEM budget (8u)");
 static_assert(kTmemColsPerSlot<P32F32F> * kNTot<P32F32F> <= kTmemCols<P32F32F>, "TMEM budget (32f)");
 static_assert(kTmemColsPerSlot<P64F64F> * kNTot<P64F64F> <= kTmemCols<P64F64F>, "TMEM budget (64f)");
+static_assert(kTmemColsPerSlot<P8U32F> * kNTot<P8U32F> <= kTmemCols<P8U32F>, "TMEM budget (8u32f)");
 
 struct KParams {
   const char* in;       // generic-path input base (TMA path uses the tensor map)
@@ -635,6 +645,42 @@ __device__ __forceinline__ void rows_scan(const float* tile, int lane, float (&r
   }
 }
 
+// 8u -> 32f: each lane's 4 bytes widened to fp32 (exact), then the 32f scan.
+template <int RW>
+__device__ __forceinline__ void rows_scan(const uint8_t* tile, int lane, float (&rowcarry)[RW],
+                                          float (&R)[RW][1][4]) {
+  constexpr int TW = 128;
+  float p[RW][4], inc[RW];
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const uint32_t b = *reinterpret_cast<const uint32_t*>(tile + i * TW + 4 * lane);
+    p[i][0] = (float)(b & 0xffu);  // Alg. 2
+    p[i][1] = p[i][0] + (float)((b >> 8) & 0xffu);
+    p[i][2] = p[i][1] + (float)((b >> 16) & 0xffu);
+    p[i][3] = p[i][2] + (float)(b >> 24);
+    inc[i] = p[i][3];
+  }
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {  // Alg. 3
+    float o[RW];
+#pragma unroll
+    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+      if (lane >= d) inc[i] += o[i];
+  }
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const float tot = __shfl_sync(kFull, inc[i], 31);
+    float ex = __shfl_up_sync(kFull, inc[i], 1);
+    if (lane == 0) ex = 0.0f;
+    const float base = rowcarry[i] + ex;
+    rowcarry[i] += tot;
+#pragma unroll
+    for (int e = 0; e < 4; ++e) R[i][0][e] = base + p[i][e];
+  }
+}
+
 template <int RW>
 __device__ __forceinline__ void rows_scan(const double* tile, int lane, double (&rowcarry)[RW],
                                           double (&R)[RW][1][2]) {
@@ -698,6 +744,8 @@ struct Tag<P32F32F> {
     for (int e = 0; e < 4; ++e) v[e] = __uint_as_float((uint32_t)w[e]);
   }
 };
+template <>
+struct Tag<P8U32F> : Tag<P32F32F> {};
 template <>
 struct Tag<P64F64F> {
   static __device__ __forceinline__ void enc(const double (&v)[2], uint32_t t, uint64_t (&w)[4]) {

@@ -212,6 +212,7 @@ sat_status sat_rect_sums(sat_plan plan, const void* sat, int64_t h, int64_t w,
     case SAT_8U_32S:
       return launch_rects<int32_t>(sat, sat_pitch_bytes, h, w, rects, n, out, s);
     case SAT_32F_32F:
+    case SAT_8U_32F:
       return launch_rects<float>(sat, sat_pitch_bytes, h, w, rects, n, out, s);
     case SAT_64F_64F:
       return launch_rects<double>(sat, sat_pitch_bytes, h, w, rects, n, out, s);
@@ -240,6 +241,7 @@ sat_status sat_box_filter(sat_plan plan, const void* sat, void* out, int64_t h, 
     case SAT_8U_32S:
       return launch_box<int32_t>(sat, out, h, w, sat_pitch_bytes, out_pitch_bytes, ry, rx, s);
     case SAT_32F_32F:
+    case SAT_8U_32F:
       return launch_box<float>(sat, out, h, w, sat_pitch_bytes, out_pitch_bytes, ry, rx, s);
     case SAT_64F_64F:
       return launch_box<double>(sat, out, h, w, sat_pitch_bytes, out_pitch_bytes, ry, rx, s);

@@ -36,13 +36,27 @@ sat_status cuda_fail(cudaError_t e, const char* what) {
               what, cudaGetErrorName(e), cudaGetErrorString(e));
 }
 
-size_t in_size(sat_pair p) { return p == SAT_8U_32S ? 1 : (p == SAT_32F_32F ? 4 : 8); }
+size_t in_size(sat_pair p) {
+  return (p == SAT_8U_32S || p == SAT_8U_32F) ? 1 : (p == SAT_32F_32F ? 4 : 8);
+}
 size_t out_size(sat_pair p) { return p == SAT_64F_64F ? 8 : 4; }
 int tile_w(sat_pair p) {
-  return p == SAT_8U_32S ? Cfg<P8U32S>::TW : (p == SAT_32F_32F ? Cfg<P32F32F>::TW : Cfg<P64F64F>::TW);
+  switch (p) {
+    case SAT_8U_32S: return Cfg<P8U32S>::TW;
+    case SAT_32F_32F: return Cfg<P32F32F>::TW;
+    case SAT_64F_64F: return Cfg<P64F64F>::TW;
+    case SAT_8U_32F: return Cfg<P8U32F>::TW;
+  }
+  return 1;
 }
 int tile_h(sat_pair p) {
-  return p == SAT_8U_32S ? Cfg<P8U32S>::TH : (p == SAT_32F_32F ? Cfg<P32F32F>::TH : Cfg<P64F64F>::TH);
+  switch (p) {
+    case SAT_8U_32S: return Cfg<P8U32S>::TH;
+    case SAT_32F_32F: return Cfg<P32F32F>::TH;
+    case SAT_64F_64F: return Cfg<P64F64F>::TH;
+    case SAT_8U_32F: return Cfg<P8U32F>::TH;
+  }
+  return 1;
 }
 
 // ---------------------------------------------------------------------------
@@ -102,7 +116,8 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   if (tma) {
     EncodeTiledFn enc = get_encode();
     if (!enc) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
-    const CUtensorMapDataType dt = kBase<P> == P8U32S    ? CU_TENSOR_MAP_DATA_TYPE_UINT8
+    const CUtensorMapDataType dt = (kBase<P> == P8U32S || kBase<P> == P8U32F)
+                                       ? CU_TENSOR_MAP_DATA_TYPE_UINT8
                                    : kBase<P> == P32F32F ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
                                                   : CU_TENSOR_MAP_DATA_TYPE_FLOAT64;
     cuuint64_t dims[3] = {(cuuint64_t)w, (cuuint64_t)h, (cuuint64_t)batch};
@@ -265,6 +280,8 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
         return launch_t<P32F32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
       case SAT_64F_64F:
         return launch_t<P64F64F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+      case SAT_8U_32F:
+        return launch_t<P8U32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
     }
   }
   switch (pl->pair) {
@@ -274,6 +291,8 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
       return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
     case SAT_64F_64F:
       return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+    case SAT_8U_32F:
+      return launch_t<P8U32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
@@ -382,6 +401,8 @@ sat_status configure(sat_plan_st* pl) {
       return configure_t<P32F32F>(pl);
     case SAT_64F_64F:
       return configure_t<P64F64F>(pl);
+    case SAT_8U_32F:
+      return configure_t<P8U32F>(pl);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
@@ -476,7 +497,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
                            int64_t max_batch) {
   if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan out-pointer is NULL");
   *plan = nullptr;
-  if (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F)
+  if (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F && pair != SAT_8U_32F)
     return fail(SAT_ERR_INVALID_ARGUMENT, "unknown pair %d", (int)pair);
   if (max_h <= 0 || max_w <= 0 || max_batch <= 0)
     return fail(SAT_ERR_INVALID_ARGUMENT, "plan limits must be positive");

@@ -92,6 +92,12 @@ def main():
         res["entries"].append({"impl": "libsat sat_compute_exclusive (H+1)x(W+1)", "pair": "8u->32s",
                                "shape": f"{H}x{W}", "ms": ms, "gpx_s": px / ms / 1e6,
                                "alg_gbs": ws / ms / 1e6})
+        ex_f = torch.empty((H + 1, W + 4), dtype=torch.float32, device="cuda")[:, :W + 1]
+        ms = timeit(lambda: sat.sat_exclusive(x, full=True, out=ex_f), steps, ws)
+        res["entries"].append({"impl": "libsat sat_compute_exclusive 8u->32f (H+1)x(W+1)",
+                               "pair": "8u->32f", "shape": f"{H}x{W}", "ms": ms,
+                               "gpx_s": px / ms / 1e6, "alg_gbs": ws / ms / 1e6})
+        del ex_f
         if lib is not None:
             for name, dt, fn in (("nppiIntegral_8u32s_C1R", torch.int32, lib.nppiIntegral_8u32s_C1R),
                                  ("nppiIntegral_8u32f_C1R", torch.float32, lib.nppiIntegral_8u32f_C1R)):
