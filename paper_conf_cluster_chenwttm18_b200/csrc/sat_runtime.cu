@@ -148,7 +148,8 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   // bands to fill the machine (shorter look-back chains pay off there); 4 for
   // 8u->32s and for short/wide images (measured).
   const int64_t nbands = kp.total_bands;
-  int CL = (kBase<P> != P8U32S && nbands >= 264) ? 8 : 4;
+  const bool byte_in = kBase<P> == P8U32S || kBase<P> == P8U32F;
+  int CL = (!byte_in && nbands >= 264) ? 8 : 4;
   if (pl->cluster > 0) CL = pl->cluster;
   const int cl_env = getenv_int("SAT_CLUSTER", 0);
   if (cl_env == 1 || cl_env == 4 || cl_env == 8) CL = cl_env;

@@ -148,3 +148,13 @@ def test_8u32f_box_filter_on_float_sat():
     ref = oracle.box_filter(x.cpu().numpy(), 3, 5).view(np.uint32).astype(np.float64)
     err = np.max(np.abs(B.cpu().numpy().astype(np.float64) - ref))
     assert err <= 4 * TOL * float(S.max())
+
+
+def test_8u32f_host_streamed_path():
+    torch, sat = _t(), _sat()
+    xh = torch.empty((1500, 2100), dtype=torch.uint8).pin_memory()
+    xd = _img(1500, 2100, seed=307)
+    xh.copy_(xd.cpu())
+    oh = torch.empty((1500, 2100), dtype=torch.float32).pin_memory()
+    y = sat.sat_host(xh, out=oh)
+    assert _rel(y.numpy(), oracle.sat_8u32f(xh.numpy())) <= TOL
