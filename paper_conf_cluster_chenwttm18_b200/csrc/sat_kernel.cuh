@@ -124,11 +124,11 @@ struct Cfg<P64F64F> {
   static constexpr int NCW = 8;
   static constexpr int NSTAGE = 3;
 };
-// 8u -> 32f (NPP's nppiIntegral_8u32f): bytes in, the fp32 scans of 32f.
+// 8u -> 32f (NPP's nppiIntegral_8u32f): the 8u->32s geometry (256-column
+// tiles, two 4-byte lane groups), fp32 values and scans.
 template <>
-struct Cfg<P8U32F> : Cfg<P32F32F> {
-  using TA = uint8_t;
-  static constexpr int NSTAGE = 4;
+struct Cfg<P8U32F> : Cfg<P8U32S> {
+  using TB = float;
 };
 
 template <int P>
@@ -645,39 +645,53 @@ __device__ __forceinline__ void rows_scan(const float* tile, int lane, float (&r
   }
 }
 
-// 8u -> 32f: each lane's 4 bytes widened to fp32 (exact), then the 32f scan.
+// 8u -> 32f, 256-column tiles: each lane widens two 4-byte groups (columns
+// 4l.. and 128+4l..) to fp32, prefix within the group (Alg. 2), and scans the
+// two group totals across the warp (Alg. 3, one Kogge-Stone per group).
 template <int RW>
 __device__ __forceinline__ void rows_scan(const uint8_t* tile, int lane, float (&rowcarry)[RW],
-                                          float (&R)[RW][1][4]) {
-  constexpr int TW = 128;
-  float p[RW][4], inc[RW];
+                                          float (&R)[RW][2][4]) {
+  constexpr int TW = 256;
+  float p[RW][2][4], inc[RW][2];
 #pragma unroll
-  for (int i = 0; i < RW; ++i) {
-    const uint32_t b = *reinterpret_cast<const uint32_t*>(tile + i * TW + 4 * lane);
-    p[i][0] = (float)(b & 0xffu);  // Alg. 2
-    p[i][1] = p[i][0] + (float)((b >> 8) & 0xffu);
-    p[i][2] = p[i][1] + (float)((b >> 16) & 0xffu);
-    p[i][3] = p[i][2] + (float)(b >> 24);
-    inc[i] = p[i][3];
-  }
+  for (int i = 0; i < RW; ++i)
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {  // Alg. 3
-    float o[RW];
+    for (int g = 0; g < 2; ++g) {
+      const uint32_t b = *reinterpret_cast<const uint32_t*>(tile + i * TW + g * 128 + 4 * lane);
+      p[i][g][0] = (float)(b & 0xffu);
+      p[i][g][1] = p[i][g][0] + (float)((b >> 8) & 0xffu);
+      p[i][g][2] = p[i][g][1] + (float)((b >> 16) & 0xffu);
+      p[i][g][3] = p[i][g][2] + (float)(b >> 24);
+      inc[i][g] = p[i][g][3];
+    }
 #pragma unroll
-    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
+  for (int d = 1; d < 32; d <<= 1) {
+    float o[RW][2];
 #pragma unroll
     for (int i = 0; i < RW; ++i)
-      if (lane >= d) inc[i] += o[i];
+#pragma unroll
+      for (int g = 0; g < 2; ++g) o[i][g] = __shfl_up_sync(kFull, inc[i][g], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+#pragma unroll
+      for (int g = 0; g < 2; ++g)
+        if (lane >= d) inc[i][g] += o[i][g];
   }
 #pragma unroll
   for (int i = 0; i < RW; ++i) {
-    const float tot = __shfl_sync(kFull, inc[i], 31);
-    float ex = __shfl_up_sync(kFull, inc[i], 1);
-    if (lane == 0) ex = 0.0f;
-    const float base = rowcarry[i] + ex;
-    rowcarry[i] += tot;
+    const float tot0 = __shfl_sync(kFull, inc[i][0], 31);
+    const float tot1 = __shfl_sync(kFull, inc[i][1], 31);
+    float ex0 = __shfl_up_sync(kFull, inc[i][0], 1);
+    float ex1 = __shfl_up_sync(kFull, inc[i][1], 1);
+    if (lane == 0) ex0 = ex1 = 0.0f;
+    const float base0 = rowcarry[i] + ex0;
+    const float base1 = (rowcarry[i] + tot0) + ex1;
+    rowcarry[i] = (rowcarry[i] + tot0) + tot1;
 #pragma unroll
-    for (int e = 0; e < 4; ++e) R[i][0][e] = base + p[i][e];
+    for (int e = 0; e < 4; ++e) {
+      R[i][0][e] = base0 + p[i][0][e];
+      R[i][1][e] = base1 + p[i][1][e];
+    }
   }
 }
 
