@@ -212,3 +212,14 @@ def sat_8u32f(A: np.ndarray) -> np.ndarray:
     result is judged against it with the 32f bar (1e-4 relative)."""
     assert A.dtype == np.uint8
     return sat(np.ascontiguousarray(A, dtype=np.float64))
+
+
+def sat_32s(A: np.ndarray) -> np.ndarray:
+    """Reference for the 32s->32s pair: the exact inclusive sums of an int32
+    image reported mod 2^32 as int32 (reading R2, as for 8u->32s).  Sums run
+    in uint64 (numpy cumsum as the library step, Eq. 1 written as the two
+    one-dimensional prefix sums it factors into); uint64 wraps mod 2^64, so
+    the low 32 bits are exact for any size."""
+    assert A.dtype == np.int32 and A.ndim == 2
+    S = A.astype(np.int64).astype(np.uint64).cumsum(axis=0, dtype=np.uint64).cumsum(axis=1, dtype=np.uint64)
+    return (S & np.uint64(0xFFFFFFFF)).astype(np.uint32).view(np.int32)

@@ -91,3 +91,17 @@ def test_8u32f_reference_is_exact_sum():
     B = np.full((300, 70000), 255, dtype=np.uint8)  # total 5.4e9 > 2^32
     got = oracle.sat_8u32f(B)
     assert got[-1, -1] == 255.0 * 300 * 70000
+
+
+def test_32s_reference_bruteforce_and_8u_agreement():
+    """oracle.sat_32s: brute force (Python ints, negative values, reported mod
+    2^32) and equality with the independent 8u->32s recurrence oracle on
+    inputs in [0, 255] (including past 2^31 where both wrap)."""
+    A = RNG.integers(-2**31, 2**31, (5, 7), dtype=np.int64).astype(np.int32)
+    got = oracle.sat_32s(A)
+    for i in range(5):
+        for j in range(7):
+            s = int(A[:i + 1, :j + 1].astype(object).sum()) % (1 << 32)
+            assert int(got[i, j].view(np.uint32)) == s
+    B = np.full((3000, 3000), 255, dtype=np.uint8)
+    assert np.array_equal(oracle.sat_32s(B.astype(np.int32)), oracle.sat(B))
