@@ -43,9 +43,9 @@ WORKLOADS = {
     "64f-16384sq": (2, 16384, 16384, 1, 1005),
 }
 DEFAULT_WORKLOAD = "sweep-16384sq-8u32s"
-PAIR_NAME = {0: "8u->32s", 1: "32f->32f", 2: "64f->64f", 3: "8u->32f"}
-IN_B = {0: 1, 1: 4, 2: 8, 3: 1}
-OUT_B = {0: 4, 1: 4, 2: 8, 3: 4}
+PAIR_NAME = {0: "8u->32s", 1: "32f->32f", 2: "64f->64f", 3: "8u->32f", 4: "32s->32s"}
+IN_B = {0: 1, 1: 4, 2: 8, 3: 1, 4: 4}
+OUT_B = {0: 4, 1: 4, 2: 8, 3: 4, 4: 4}
 DTYPE_NAME = {0: "u32", 1: "f32", 2: "f64"}
 L2_BYTES = 126 * 1024 * 1024
 
@@ -232,10 +232,13 @@ def time_device(sat, x, out, steps, warmup, flush=None, stream=None):
 
 
 def sweep_entry(sat, satgen, torch, pair, H, W, N, seed, steps, peak):
-    dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64, 3: torch.uint8}[pair]
+    dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64, 3: torch.uint8, 4: torch.int32}[pair]
     shape = (N, H, W) if N > 1 else (H, W)
     x = torch.empty(shape, dtype=dt, device="cuda")
-    satgen.fill_device(x, seed=seed)
+    if pair == 4:  # satgen has no int32 kind: full-range torch randoms (every sum wraps)
+        x.random_(-2**31, 2**31 - 1, generator=torch.Generator(device="cuda").manual_seed(seed))
+    else:
+        satgen.fill_device(x, seed=seed)
     out = torch.empty(shape, dtype=sat.out_dtype(pair), device="cuda")
     byts = H * W * N * (IN_B[pair] + OUT_B[pair])
     flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device="cuda") if byts < 4 * L2_BYTES else None
@@ -379,7 +382,7 @@ def run_ours(args, workload, rank, world, local_rank):
                                  (1, 8192, 8192, 1), (1, 16384, 16384, 1), (2, 16384, 16384, 1),
                                  (2, 4096, 65536, 1), (2, 65536, 4096, 1), (0, 4096, 65536, 1),
                                  (1, 65536, 4096, 1), (0, 1080, 1920, 1024),
-                                 (1, 65536, 65536, 1), (3, 16384, 16384, 1)]:
+                                 (1, 65536, 65536, 1), (3, 16384, 16384, 1), (4, 16384, 16384, 1)]:
             try:
                 sweep.append(sweep_entry(sat, satgen, torch, p_, h_, w_, n_, 1001, 10, peak))
             except Exception as ex:  # e.g. OOM: report, keep going

@@ -11,6 +11,8 @@
  *     SAT_32F_32F : float  -> float  (accumulated in fp32; tolerance 1e-4 rel.)
  *     SAT_64F_64F : double -> double (accumulated in fp64; tolerance 1e-12 rel.)
  *     SAT_8U_32F  : uint8  -> float  (accumulated in fp32; tolerance 1e-4 rel.)
+ *     SAT_32S_32S : int32  -> int32, exact, two's-complement wrap mod 2^32
+ * (8u->32u is SAT_8U_32S's output read as uint32: the same bits mod 2^32.)
  * Output has the same h x w shape as the input (inclusive form).
  *
  * Conventions (all entry points):
@@ -63,7 +65,7 @@ typedef enum {
 /* Type pairs T_A -> T_B.  SAT_8U_32F is NPP's second pair
  * (nppiIntegral_8u32f): uint8 input, float output accumulated in
  * fp32 (tolerance 1e-4 relative to the exact sum, as for 32f). */
-typedef enum { SAT_8U_32S = 0, SAT_32F_32F = 1, SAT_64F_64F = 2, SAT_8U_32F = 3 } sat_pair;
+typedef enum { SAT_8U_32S = 0, SAT_32F_32F = 1, SAT_64F_64F = 2, SAT_8U_32F = 3, SAT_32S_32S = 4 } sat_pair;
 
 typedef struct sat_plan_st* sat_plan;
 typedef struct sat_comm_st* sat_comm;

@@ -17,9 +17,10 @@ import os
 import threading
 
 __all__ = ["SatError", "Plan", "sat", "sat_host", "SatComm", "sat_dist", "band_partition",
-           "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "PAIR_8U_32F", "lib", "LIB_PATH"]
+           "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "PAIR_8U_32F", "PAIR_32S_32S", "lib",
+           "LIB_PATH"]
 
-PAIR_8U_32S, PAIR_32F_32F, PAIR_64F_64F, PAIR_8U_32F = 0, 1, 2, 3
+PAIR_8U_32S, PAIR_32F_32F, PAIR_64F_64F, PAIR_8U_32F, PAIR_32S_32S = 0, 1, 2, 3, 4
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("SAT_LIBRARY") or os.path.join(_HERE, "libsat.so")
 COMM_ID_BYTES = 128
@@ -94,9 +95,10 @@ def _torch():
 def pair_of_dtype(dtype, out=None) -> int:
     """Type pair of an input dtype; uint8 with a float32 output is 8u->32f."""
     torch = _torch()
-    m = {torch.uint8: PAIR_8U_32S, torch.float32: PAIR_32F_32F, torch.float64: PAIR_64F_64F}
+    m = {torch.uint8: PAIR_8U_32S, torch.float32: PAIR_32F_32F, torch.float64: PAIR_64F_64F,
+         torch.int32: PAIR_32S_32S}
     if dtype not in m:
-        raise TypeError(f"unsupported input dtype {dtype}; expected uint8, float32 or float64")
+        raise TypeError(f"unsupported input dtype {dtype}; expected uint8, int32, float32 or float64")
     if dtype == torch.uint8 and out == torch.float32:
         return PAIR_8U_32F
     return m[dtype]
@@ -105,7 +107,7 @@ def pair_of_dtype(dtype, out=None) -> int:
 def out_dtype(pair: int):
     torch = _torch()
     return {PAIR_8U_32S: torch.int32, PAIR_32F_32F: torch.float32, PAIR_64F_64F: torch.float64,
-            PAIR_8U_32F: torch.float32}[pair]
+            PAIR_8U_32F: torch.float32, PAIR_32S_32S: torch.int32}[pair]
 
 
 _out_dtype_of = out_dtype  # for functions whose `out_dtype` parameter shadows the helper
@@ -253,7 +255,8 @@ def sat_exclusive(x, full: bool = True, nval=0, out=None, plan: Plan | None = No
         raise ValueError("out has the wrong dtype/shape/device")
     if out.numel() == 0:
         return out
-    ctype = {0: ctypes.c_int32, 1: ctypes.c_float, 2: ctypes.c_double, 3: ctypes.c_float}[pair]
+    ctype = {0: ctypes.c_int32, 1: ctypes.c_float, 2: ctypes.c_double, 3: ctypes.c_float,
+             4: ctypes.c_int32}[pair]
     nv = ctype(nval)
     ip = _row_layout(x)[0] if H > 0 and W > 0 else max(W, 1) * x.element_size()
     op = _row_layout(out)[0]
@@ -415,7 +418,7 @@ def dist_colsum(band, plan: Plan | None = None, stream=None, pair=None):
     torch = _torch()
     pair = pair_of_dtype(band.dtype) if pair is None else pair
     H, W = band.shape
-    acc = torch.empty(W, dtype=torch.int32 if pair == PAIR_8U_32S else torch.float64, device=band.device)
+    acc = torch.empty(W, dtype=torch.int32 if pair in (PAIR_8U_32S, PAIR_32S_32S) else torch.float64, device=band.device)
     ip = band.stride(0) * band.element_size() if H > 1 else W * band.element_size()
     p = plan if plan is not None else _plan_for(band.device, pair, max(H, 1), W, 1)
     _check(lib().sat_dist_colsum(p.handle, band.data_ptr() if H else None, H, W, ip,

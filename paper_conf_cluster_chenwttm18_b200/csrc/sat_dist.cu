@@ -221,7 +221,7 @@ __global__ void sat_carry_finish_kernel(const ACC* __restrict__ local, const ACC
   if (x < w) carry[x] = (TB)(tile_off[x / kCarryTile] + local[x]);
 }
 
-size_t acc_size(sat_pair p) { return p == SAT_8U_32S ? 4 : 8; }
+size_t acc_size(sat_pair p) { return (p == SAT_8U_32S || p == SAT_32S_32S) ? 4 : 8; }
 
 // ---------------------------------------------------------------------------
 
@@ -262,6 +262,10 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
         sat_colsum_vec_kernel<uint8_t, double, 4><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
         sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
         break;
+      case SAT_32S_32S:
+        sat_colsum_vec_kernel<uint32_t, uint32_t, 4><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (uint32_t*)partial);
+        sat_colsum_reduce_kernel<uint32_t><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((uint32_t*)partial, used, w, (uint32_t*)out);
+        break;
       case SAT_64F_64F:
         sat_colsum_vec_kernel<double, double, 2><<<gv, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
         sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
@@ -283,6 +287,10 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
       sat_colsum_kernel<uint8_t, double><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
       sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
       break;
+    case SAT_32S_32S:
+      sat_colsum_kernel<uint32_t, uint32_t><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (uint32_t*)partial);
+      sat_colsum_reduce_kernel<uint32_t><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((uint32_t*)partial, used, w, (uint32_t*)out);
+      break;
     case SAT_64F_64F:
       sat_colsum_kernel<double, double><<<grid, kColsumThreads, 0, s>>>(p, h, w, pitch, rps, (double*)partial);
       sat_colsum_reduce_kernel<double><<<(unsigned)((w + 255) / 256), 256, 0, s>>>((double*)partial, used, w, (double*)out);
@@ -301,7 +309,8 @@ sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, 
   if (e != cudaSuccess) return cuda_fail(e, "cudaMallocAsync(carry scratch)");
   const unsigned fin = (unsigned)((w + 255) / 256);
   switch (pair) {
-    case SAT_8U_32S: {
+    case SAT_8U_32S:
+    case SAT_32S_32S: {
       uint32_t* loc = (uint32_t*)scratch;
       uint32_t* tt = loc + w;
       sat_carry_scan_kernel<uint32_t><<<(unsigned)ntiles, kCarryThreads, 0, s>>>((const uint32_t*)gathered, rank, w, loc, tt);
@@ -490,7 +499,7 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
   if (st != SAT_OK) return st;
   st = colsum(pair, in_band, band_h, w, in_pitch_bytes, b.partial, b.splits, b.local, s);
   if (st != SAT_OK) return st;
-  const ncclDataType_t dt = pair == SAT_8U_32S ? ncclUint32 : ncclFloat64;
+  const ncclDataType_t dt = acc_size(pair) == 4 ? ncclUint32 : ncclFloat64;
   ncclResult_t r = nccl().AllGather(b.local, b.gathered, (size_t)w, dt, comm->comm, s);
   if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
   st = band_carry(pair, b.gathered, comm->rank, w, b.carry, s);
@@ -504,7 +513,7 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
 
 size_t sat_chain_bytes(sat_pair pair, int64_t w) {
   if (w <= 0 || (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F &&
-                 pair != SAT_8U_32F))
+                 pair != SAT_8U_32F && pair != SAT_32S_32S))
     return 0;
   // one tagged 64-bit word per 32-bit half of each output element, per chunk
   const int64_t tw = tile_w(pair);

@@ -16,8 +16,8 @@ struct sat_plan_st {
   sat_pair pair = SAT_8U_32S;
   int64_t max_h = 0, max_w = 0, max_batch = 0;
   int num_sms = 0;
-  int active_clusters[4][3][4] = {};  // [pair][cluster 1/4/8][mode: bit0 TMA, bit1 vec out]
-  int active_short[4] = {};           // [pair] short-band variant, clusters of 4, TMA + vec out
+  int active_clusters[5][3][4] = {};  // [pair][cluster 1/4/8][mode: bit0 TMA, bit1 vec out]
+  int active_short[5] = {};           // [pair] short-band variant, clusters of 4, TMA + vec out
   int cluster = 0;                    // forced CTAs (bands) per cluster (0: by shape)
   int64_t max_tiles = 0;       // capacity of the look-back workspace in tiles
   void* ws = nullptr;

@@ -57,11 +57,11 @@
 
 namespace sat {
 
-enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2, P8U32F = 3 };
+enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2, P8U32F = 3, P32S32S = 4 };
 // Short-band variants (P + kShort): the same pair with 16-row bands (2 rows per
 // compute warp), chosen for short, wide images whose 32-row bands would leave
 // most of the machine idle (H / 4 compute warps in total otherwise).
-constexpr int kShort = 4;
+constexpr int kShort = 5;
 template <int P>
 constexpr int kBase = P % kShort;
 
@@ -130,6 +130,12 @@ template <>
 struct Cfg<P8U32F> : Cfg<P8U32S> {
   using TB = float;
 };
+// 32s -> 32s: the 32f geometry with wrap-around u32 integer scans (R2).
+template <>
+struct Cfg<P32S32S> : Cfg<P32F32F> {
+  using TA = uint32_t;
+  using TB = uint32_t;
+};
 
 template <int P>
 struct CfgShort : Cfg<P> {
@@ -143,6 +149,8 @@ template <>
 struct Cfg<P64F64F + kShort> : CfgShort<P64F64F> {};
 template <>
 struct Cfg<P8U32F + kShort> : CfgShort<P8U32F> {};
+template <>
+struct Cfg<P32S32S + kShort> : CfgShort<P32S32S> {};
 
 
 // Warp roles: NCW compute warps, then the producer, then kNLB look-back warps.
@@ -186,6 +194,7 @@ static_assert(kTmemColsPerSlot<P8U32S> * kNTot<P8U32S> <= kTmemCols<P8U32S>, "TM
 static_assert(kTmemColsPerSlot<P32F32F> * kNTot<P32F32F> <= kTmemCols<P32F32F>, "TMEM budget (32f)");
 static_assert(kTmemColsPerSlot<P64F64F> * kNTot<P64F64F> <= kTmemCols<P64F64F>, "TMEM budget (64f)");
 static_assert(kTmemColsPerSlot<P8U32F> * kNTot<P8U32F> <= kTmemCols<P8U32F>, "TMEM budget (8u32f)");
+static_assert(kTmemColsPerSlot<P32S32S> * kNTot<P32S32S> <= kTmemCols<P32S32S>, "TMEM budget (32s)");
 
 struct KParams {
   const char* in;       // generic-path input base (TMA path uses the tensor map)
@@ -695,6 +704,40 @@ __device__ __forceinline__ void rows_scan(const uint8_t* tile, int lane, float (
   }
 }
 
+// 32s -> 32s: as the 32f scan, in wrap-around uint32 arithmetic (exact mod 2^32).
+template <int RW>
+__device__ __forceinline__ void rows_scan(const uint32_t* tile, int lane, uint32_t (&rowcarry)[RW],
+                                          uint32_t (&R)[RW][1][4]) {
+  constexpr int TW = 128;
+  uint32_t p[RW][4], inc[RW];
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const uint4 a = *reinterpret_cast<const uint4*>(tile + i * TW + 4 * lane);
+    p[i][0] = a.x;  // Alg. 2
+    p[i][1] = p[i][0] + a.y;
+    p[i][2] = p[i][1] + a.z;
+    p[i][3] = p[i][2] + a.w;
+    inc[i] = p[i][3];
+  }
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {  // Alg. 3
+    uint32_t o[RW];
+#pragma unroll
+    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+      if (lane >= d) inc[i] += o[i];
+  }
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const uint32_t tot = __shfl_sync(kFull, inc[i], 31);
+    const uint32_t base = rowcarry[i] + (inc[i] - p[i][3]);
+    rowcarry[i] += tot;
+#pragma unroll
+    for (int e = 0; e < 4; ++e) R[i][0][e] = base + p[i][e];
+  }
+}
+
 template <int RW>
 __device__ __forceinline__ void rows_scan(const double* tile, int lane, double (&rowcarry)[RW],
                                           double (&R)[RW][1][2]) {
@@ -760,6 +803,8 @@ struct Tag<P32F32F> {
 };
 template <>
 struct Tag<P8U32F> : Tag<P32F32F> {};
+template <>
+struct Tag<P32S32S> : Tag<P8U32S> {};
 template <>
 struct Tag<P64F64F> {
   static __device__ __forceinline__ void enc(const double (&v)[2], uint32_t t, uint64_t (&w)[4]) {

@@ -210,6 +210,7 @@ sat_status sat_rect_sums(sat_plan plan, const void* sat, int64_t h, int64_t w,
   }
   switch (pair) {
     case SAT_8U_32S:
+    case SAT_32S_32S:
       return launch_rects<int32_t>(sat, sat_pitch_bytes, h, w, rects, n, out, s);
     case SAT_32F_32F:
     case SAT_8U_32F:
@@ -239,6 +240,7 @@ sat_status sat_box_filter(sat_plan plan, const void* sat, void* out, int64_t h, 
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   switch (pair) {
     case SAT_8U_32S:
+    case SAT_32S_32S:
       return launch_box<int32_t>(sat, out, h, w, sat_pitch_bytes, out_pitch_bytes, ry, rx, s);
     case SAT_32F_32F:
     case SAT_8U_32F:

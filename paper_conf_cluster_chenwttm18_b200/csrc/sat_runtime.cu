@@ -37,7 +37,7 @@ sat_status cuda_fail(cudaError_t e, const char* what) {
 }
 
 size_t in_size(sat_pair p) {
-  return (p == SAT_8U_32S || p == SAT_8U_32F) ? 1 : (p == SAT_32F_32F ? 4 : 8);
+  return (p == SAT_8U_32S || p == SAT_8U_32F) ? 1 : (p == SAT_64F_64F ? 8 : 4);
 }
 size_t out_size(sat_pair p) { return p == SAT_64F_64F ? 8 : 4; }
 int tile_w(sat_pair p) {
@@ -46,6 +46,7 @@ int tile_w(sat_pair p) {
     case SAT_32F_32F: return Cfg<P32F32F>::TW;
     case SAT_64F_64F: return Cfg<P64F64F>::TW;
     case SAT_8U_32F: return Cfg<P8U32F>::TW;
+    case SAT_32S_32S: return Cfg<P32S32S>::TW;
   }
   return 1;
 }
@@ -55,6 +56,7 @@ int tile_h(sat_pair p) {
     case SAT_32F_32F: return Cfg<P32F32F>::TH;
     case SAT_64F_64F: return Cfg<P64F64F>::TH;
     case SAT_8U_32F: return Cfg<P8U32F>::TH;
+    case SAT_32S_32S: return Cfg<P32S32S>::TH;
   }
   return 1;
 }
@@ -119,6 +121,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
     const CUtensorMapDataType dt = (kBase<P> == P8U32S || kBase<P> == P8U32F)
                                        ? CU_TENSOR_MAP_DATA_TYPE_UINT8
                                    : kBase<P> == P32F32F ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                   : kBase<P> == P32S32S ? CU_TENSOR_MAP_DATA_TYPE_UINT32
                                                   : CU_TENSOR_MAP_DATA_TYPE_FLOAT64;
     cuuint64_t dims[3] = {(cuuint64_t)w, (cuuint64_t)h, (cuuint64_t)batch};
     cuuint64_t strides[2] = {(cuuint64_t)ip, (cuuint64_t)(batch > 1 ? iis : ip * h)};
@@ -283,6 +286,8 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
         return launch_t<P64F64F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
       case SAT_8U_32F:
         return launch_t<P8U32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+      case SAT_32S_32S:
+        return launch_t<P32S32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
     }
   }
   switch (pl->pair) {
@@ -294,6 +299,8 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
       return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
     case SAT_8U_32F:
       return launch_t<P8U32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+    case SAT_32S_32S:
+      return launch_t<P32S32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
@@ -404,6 +411,8 @@ sat_status configure(sat_plan_st* pl) {
       return configure_t<P64F64F>(pl);
     case SAT_8U_32F:
       return configure_t<P8U32F>(pl);
+    case SAT_32S_32S:
+      return configure_t<P32S32S>(pl);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
@@ -498,7 +507,8 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
                            int64_t max_batch) {
   if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan out-pointer is NULL");
   *plan = nullptr;
-  if (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F && pair != SAT_8U_32F)
+  if (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F && pair != SAT_8U_32F &&
+      pair != SAT_32S_32S)
     return fail(SAT_ERR_INVALID_ARGUMENT, "unknown pair %d", (int)pair);
   if (max_h <= 0 || max_w <= 0 || max_batch <= 0)
     return fail(SAT_ERR_INVALID_ARGUMENT, "plan limits must be positive");
