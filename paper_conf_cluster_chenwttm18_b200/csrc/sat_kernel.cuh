@@ -1,7 +1,12 @@
 // sat_kernel.cuh -- single-pass summed-area-table kernel for sm_100a.
 //
 // What it computes: the inclusive SAT S(i,j) = sum_{y<=i, x<=j} A(y,x)
-// (Eq. 1) of pitched row-major images, in one HBM pass.
+// (Eq. 1) of pitched row-major images, in one HBM pass, for
+// the pairs 8u->32s, 32f->32f, 64f->64f (BASELINE north star), 8u->32f and
+// 32s->32s (Cfg<P>; P + kShort = the same pair with 16-row bands).  The same
+// kernel also stores the exclusive layout (Eq. 2, template flag kEx: shifted
+// 16-byte stores) and chains bands through per-chunk carry vectors
+// (KParams::chain_in / chain_out; the single-pass multi-GPU building block).
 //
 // Decomposition: the image is cut into
 // row BANDS of TH rows; a band is walked left-to-right in CHUNKS of TW columns
