@@ -43,8 +43,8 @@ WORKLOAD_OF = {  # prof_one args -> bench workload name
     "p1_65536x65536x1": "huge-65536sq-32f32f",
     "p2_16384x16384x1": "64f-16384sq",
 }
-IN_B = {0: 1, 1: 4, 2: 8}
-OUT_B = {0: 4, 1: 4, 2: 8}
+IN_B = {0: 1, 1: 4, 2: 8, 3: 1, 4: 4}
+OUT_B = {0: 4, 1: 4, 2: 8, 3: 4, 4: 4}
 
 
 def raw(rep):

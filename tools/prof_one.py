@@ -10,10 +10,13 @@ import paper_conf_cluster_chenwttm18_b200 as sat
 import satgen
 
 pair, H, W, N, reps = (int(v) for v in sys.argv[1:6])
-dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64}[pair]
+dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64, 3: torch.uint8, 4: torch.int32}[pair]
 shape = (N, H, W) if N > 1 else (H, W)
 x = torch.empty(shape, dtype=dt, device="cuda")
-satgen.fill_device(x, seed=1)
+if pair == 4:
+    x.random_(-2**31, 2**31 - 1)
+else:
+    satgen.fill_device(x, seed=1)
 y = torch.empty(shape, dtype=sat.out_dtype(pair), device="cuda")
 for _ in range(reps):
     sat.sat(x, out=y)
