@@ -8,7 +8,14 @@ the extension is missing or the device is not a B200 the calls raise.
     S(i, j) = sum_{y <= i} sum_{x <= j} A(y, x)        (PAPER.md:58-61, Eq. 1)
 
 Type pairs: uint8 -> int32 (wrap mod 2^32), float32 -> float32,
-float64 -> float64.
+float64 -> float64; also uint8 -> float32 (``out_dtype=torch.float32``, NPP's
+8u32f) and int32 -> int32 (wrap mod 2^32).
+
+Entry points: ``sat`` (single / batched), ``sat_exclusive`` (Eq. 2 and the
+NPP (H+1) x (W+1) layout), ``sat_band`` (carry-in row), ``sat_host`` (host in,
+host out), ``sat_dist`` / ``sat_dist_chained`` (row bands across ranks),
+``sat_band_chained`` (one band of a chain), ``rect_sums`` / ``box_filter``
+(SAT consumers).
 """
 from __future__ import annotations
 
@@ -16,7 +23,9 @@ import ctypes
 import os
 import threading
 
-__all__ = ["SatError", "Plan", "sat", "sat_host", "SatComm", "sat_dist", "band_partition",
+__all__ = ["SatError", "Plan", "sat", "sat_host", "sat_exclusive", "sat_band", "SatComm", "sat_dist",
+           "sat_dist_chained", "sat_band_chained", "new_chain_buffer", "chain_bytes", "rect_sums",
+           "box_filter", "band_partition",
            "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "PAIR_8U_32F", "PAIR_32S_32S", "lib",
            "LIB_PATH"]
 
