@@ -35,6 +35,10 @@ __device__ __forceinline__ void tma_store_2d(const CUtensorMap* m, const void* s
 __device__ __forceinline__ void bulk_store(void* g, const void* s, uint32_t n) {
   asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(g), "r"(smem_u32(s)), "r"(n) : "memory");
 }
+__device__ __forceinline__ void st_cs8(void* p, uint4 a, uint4 b) {
+  asm volatile("st.global.cs.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(a.x), "r"(a.y), "r"(a.z), "r"(a.w),
+               "r"(b.x), "r"(b.y), "r"(b.z), "r"(b.w) : "memory");
+}
 __device__ __forceinline__ void st_cs(void* p, uint4 v) {
   asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
@@ -88,6 +92,13 @@ __global__ void __launch_bounds__((NW + 1) * 32) skel(const __grid_constant__ CU
     const int band = s.band[st], chunk = s.chunk[st];
     if (band < 0) break;
     uint32_t w[RW][2];
+    if (MODE == 3) {
+#pragma unroll
+      for (int i = 0; i < RW; ++i) {
+        const uint2 v = *reinterpret_cast<const uint2*>(&s.in[st][warp * RW + i][8 * lane]);
+        w[i][0] = v.x; w[i][1] = v.y;
+      }
+    } else
 #pragma unroll
     for (int i = 0; i < RW; ++i) {
       w[i][0] = *reinterpret_cast<const uint32_t*>(&s.in[st][warp * RW + i][4 * lane]);
@@ -96,7 +107,14 @@ __global__ void __launch_bounds__((NW + 1) * 32) skel(const __grid_constant__ CU
     __syncwarp();
     if (lane == 0) mbar_arrive(&s.empty[st]);
     const int64_t y0 = (int64_t)band * 32 + warp * RW, x0 = (int64_t)chunk * TW;
-    if (MODE == 0) {
+    if (MODE == 3) {
+#pragma unroll
+      for (int i = 0; i < RW; ++i) {
+        const uint32_t u = w[i][0], v = w[i][1];
+        st_cs8(p.out + (y0 + i) * p.W + x0 + 8 * lane, make_uint4(u & 255, (u >> 8) & 255, (u >> 16) & 255, u >> 24),
+               make_uint4(v & 255, (v >> 8) & 255, (v >> 16) & 255, v >> 24));
+      }
+    } else if (MODE == 0) {
 #pragma unroll
       for (int i = 0; i < RW; ++i)
 #pragma unroll
@@ -127,7 +145,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) skel(const __grid_constant__ CU
       }
     }
   }
-  if (MODE != 0 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  if (MODE != 0 && MODE != 3 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 
 typedef CUresult (*Enc)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -171,9 +189,13 @@ int main() {
     }
   };
   run(skel<8, 0>, 8, 4, "direct st.cs.v4");
+  run(skel<8, 3>, 8, 4, "direct st.cs.v8 (256-bit)");
+  run(skel<8, 0>, 8, 4, "direct st.cs.v4");
+  run(skel<8, 3>, 8, 4, "direct st.cs.v8 (256-bit)");
   run(skel<8, 1>, 8, 4, "bulk 1D per row");
   run(skel<8, 2>, 8, 4, "tensor 2D per warp");
   run(skel<16, 0>, 16, 2, "direct st.cs.v4");
+  run(skel<16, 3>, 16, 2, "direct st.cs.v8 (256-bit)");
   run(skel<16, 1>, 16, 2, "bulk 1D per row");
   run(skel<16, 2>, 16, 2, "tensor 2D per warp");
   run(skel<4, 0>, 4, 8, "direct st.cs.v4");
