@@ -97,7 +97,10 @@ struct Cfg<P8U32S> {
 #endif
   static constexpr int NCW = SAT_NCW8;   // compute warps, 4 rows each
   static constexpr int TH = 4 * NCW;     // 32 (2 CTAs per SM) or 64 (1 CTA per SM, 16 warps)
-  static constexpr int NSTAGE = 4;       // TMA prefetch depth (stages free after pass A)
+#ifndef SAT_NST8
+#define SAT_NST8 4
+#endif
+  static constexpr int NSTAGE = SAT_NST8;  // TMA prefetch depth (stages free after pass A)
 };
 template <>
 struct Cfg<P32F32F> {
@@ -112,7 +115,10 @@ struct Cfg<P32F32F> {
 #endif
   static constexpr int LOOK = SAT_LOOK32;
   static constexpr int NCW = 8;
-  static constexpr int NSTAGE = 3;
+#ifndef SAT_NST32
+#define SAT_NST32 3
+#endif
+  static constexpr int NSTAGE = SAT_NST32;
 };
 template <>
 struct Cfg<P64F64F> {
