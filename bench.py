@@ -351,7 +351,10 @@ def run_ours(args, workload, rank, world, local_rank):
 
     banded = None
     if world > 1 or args.banded:
-        banded = run_banded(args, rank, world, local_rank)
+        try:
+            banded = run_banded(args, rank, world, local_rank)
+        except Exception as ex:  # report it on the line; the headline above stands
+            banded = {"workload": "huge-65536sq-32f32f row-banded", "error": str(ex)[:300]}
 
     if rank != 0:
         return
