@@ -152,7 +152,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   // 8u->32s and for short/wide images (measured).
   const int64_t nbands = kp.total_bands;
   const bool byte_in = kBase<P> == P8U32S || kBase<P> == P8U32F;
-  int CL = (!byte_in && nbands >= 264) ? 8 : 4;
+  int CL = (!byte_in && nbands >= 224) ? 8 : 4;
   if (pl->cluster > 0) CL = pl->cluster;
   const int cl_env = getenv_int("SAT_CLUSTER", 0);
   if (cl_env == 1 || cl_env == 4 || cl_env == 8) CL = cl_env;
