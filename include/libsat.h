@@ -30,10 +30,18 @@
  *    synchronously, enqueue on `stream` (a cudaStream_t passed as void*;
  *    NULL = legacy default stream) and return without synchronising the host.
  *    Asynchronous device faults surface at the caller's next synchronisation.
- *  - A plan owns a workspace (look-back status words, carry payloads, a
- *    ticket counter).  A plan must not be used by two unordered streams at
- *    once (documented, not detected).  Workspace is never re-zeroed per call:
- *    status words carry a per-call epoch.
+ *  - A plan owns a workspace (look-back carry vectors, a ticket counter, an
+ *    error word).  Launches of one plan are ordered: a launch on a stream
+ *    other than the plan's previous one first waits (cudaStreamWaitEvent) for
+ *    that launch, so two streams sharing a plan serialise instead of racing on
+ *    the workspace.  Workspace is never re-zeroed per call: carry words carry a
+ *    per-call epoch.  Stream capture (CUDA graphs) of a compute call returns
+ *    SAT_ERR_UNSUPPORTED (tickets and epochs are handed out per launch by the
+ *    host).
+ *  - Cross-CTA and cross-GPU carry waits are bounded (sat_plan_set_timeout,
+ *    default 2 s): a wait that runs out (e.g. the band above in a chain never
+ *    ran) lets the kernel finish with wrong values and records the event;
+ *    sat_plan_status() then returns SAT_ERR_TIMEOUT.
  *  - h == 0 or w == 0 (or batch == 0) is SAT_OK and a no-op.
  *  - In-place (in == out, equal pitches/strides) is allowed for 32f/64f.
  *    Any other overlap of input and output ranges is SAT_ERR_UNSUPPORTED.
@@ -59,7 +67,8 @@ typedef enum {
   SAT_ERR_UNSUPPORTED = 2,
   SAT_ERR_CUDA = 3,
   SAT_ERR_NCCL = 4,
-  SAT_ERR_OUT_OF_MEMORY = 5
+  SAT_ERR_OUT_OF_MEMORY = 5,
+  SAT_ERR_TIMEOUT = 6
 } sat_status;
 
 /* Type pairs T_A -> T_B.  SAT_8U_32F is NPP's second pair
@@ -84,6 +93,15 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
 
 /* Bytes of device workspace owned by the plan. */
 sat_status sat_plan_workspace_bytes(sat_plan plan, size_t* bytes);
+
+/* Bound (ns, > 0) on every cross-CTA / cross-GPU carry wait of later launches
+ * of `plan` (default 2e9).  Errors: INVALID_ARGUMENT (NULL plan, ns == 0). */
+sat_status sat_plan_set_timeout(sat_plan plan, uint64_t ns);
+
+/* Synchronises `stream` and reports (then clears) the plan's device error
+ * word: SAT_ERR_TIMEOUT if a bounded carry wait of an earlier launch ran out
+ * (that launch's output is wrong), SAT_OK otherwise; CUDA on a device fault. */
+sat_status sat_plan_status(sat_plan plan, void* stream);
 
 /* Free the plan and its workspace (and host-path staging buffers).  The caller
  * must ensure no work using the plan is still pending.  NULL is a no-op. */

@@ -63,6 +63,8 @@ def lib():
                     "sat_plan_create": ([ctypes.POINTER(vp), i32, i32, i64, i64, i64], i32),
                     "sat_plan_workspace_bytes": ([vp, ctypes.POINTER(sz)], i32),
                     "sat_plan_destroy": ([vp], i32),
+                    "sat_plan_set_timeout": ([vp, ctypes.c_uint64], i32),
+                    "sat_plan_status": ([vp, vp], i32),
                     "sat_compute": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_batched": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_band": ([vp, vp, vp, i64, i64, i64, i64, vp, i32, vp], i32),
@@ -84,6 +86,8 @@ def lib():
                     "sat_last_error": ([], ctypes.c_char_p),
                 }
                 for name, (args, res) in sigs.items():
+                    if not hasattr(L, name) and os.environ.get("SAT_LIBRARY"):
+                        continue  # an explicitly chosen older build (same-box A/B tools)
                     f = getattr(L, name)
                     f.argtypes = args
                     f.restype = res
@@ -150,6 +154,15 @@ class Plan:
         _check(lib().sat_plan_workspace_bytes(self._h, ctypes.byref(n)), "sat_plan_workspace_bytes")
         return n.value
 
+    def set_timeout(self, ns: int):
+        """Bound every cross-CTA / cross-GPU carry wait of later launches (ns)."""
+        _check(lib().sat_plan_set_timeout(self._h, int(ns)), "sat_plan_set_timeout")
+
+    def status(self, stream=None):
+        """Synchronise `stream`; raise SatError(SAT_ERR_TIMEOUT) if a bounded
+        carry wait of an earlier launch ran out (that output is wrong)."""
+        _check(lib().sat_plan_status(self._h, _stream_ptr(stream, self.device)), "sat_plan_status")
+
     def close(self):
         if getattr(self, "_h", None) is not None and self._h.value:
             lib().sat_plan_destroy(self._h)
@@ -189,8 +202,13 @@ class Plan:
 _plans: dict = {}
 
 
+_KNOBS = ("SAT_FORCE_GENERIC", "SAT_CLUSTER", "SAT_SHORT", "SAT_MAX_CLUSTERS", "SAT_FORCE_CLUSTERS",
+          "SAT_LOG")
+
+
 def _plan_for(device, pair, h, w, batch) -> Plan:
-    key = (device.index, pair)
+    # libsat reads its tuning knobs once per plan: plans are cached per knob setting
+    key = (device.index, pair, tuple(os.environ.get(k) for k in _KNOBS))
     p = _plans.get(key)
     if p is None or not p.fits(h, w, batch):
         if p is not None:

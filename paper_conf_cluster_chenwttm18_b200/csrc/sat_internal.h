@@ -16,17 +16,33 @@ struct sat_plan_st {
   sat_pair pair = SAT_8U_32S;
   int64_t max_h = 0, max_w = 0, max_batch = 0;
   int num_sms = 0;
-  int active_clusters[5][3][4] = {};  // [pair][cluster 1/4/8][mode: bit0 TMA, bit1 vec out]
+  int active_clusters[5][3][4] = {};  // [pair][cluster 2/4/8][mode: bit0 TMA, bit1 vec out]
   int active_short[5] = {};           // [pair] short-band variant, clusters of 4, TMA + vec out
-  int cluster = 0;                    // forced CTAs (bands) per cluster (0: by shape)
-  int64_t max_tiles = 0;       // capacity of the look-back workspace in tiles
+  // Tuning / diagnosis knobs, read from the environment ONCE at plan creation
+  // (SAT_FORCE_GENERIC, SAT_CLUSTER, SAT_SHORT, SAT_MAX_CLUSTERS,
+  // SAT_FORCE_CLUSTERS, SAT_LOG); launches never consult the environment.
+  int force_generic = 0;
+  int cluster = 0;        // forced CTAs (bands) per cluster: 0 = by shape, else 2 / 4 / 8
+  int short_bands = -1;   // -1 by shape, 0 / 1 forced
+  int max_clusters = 0, force_clusters = 0;
+  int log = 0;
+  int64_t max_tiles = 0;       // max_batch * bands * chunks of the plan limits (normal bands)
+  int64_t tickets_cap = 0;     // cluster tickets the look-back payload holds at the plan's max width
+  int64_t max_chunks = 0;
   void* ws = nullptr;
   size_t ws_bytes = 0;
   unsigned long long* counter = nullptr;  // ticket counter
-  void* payload = nullptr;                // aggregate / inclusive carries
+  uint32_t* err = nullptr;                // device error word (bit 0: a bounded wait timed out)
+  void* payload = nullptr;                // aggregate / inclusive carry vectors
+  uint64_t spin_ns = 2000000000ull;       // bounded-wait limit (sat_plan_set_timeout)
   uint32_t epoch = 0;
   uint64_t ticket_base = 0;
   uint64_t launches = 0;
+  // Launch ordering across streams: the workspace is shared by every launch of
+  // the plan, so a launch on a different stream first waits for the previous one.
+  cudaEvent_t last_ev = nullptr;
+  cudaStream_t last_stream = nullptr;
+  bool has_last = false;
   // streamed host path (lazily allocated)
   sat::HostPath* host = nullptr;
 };
@@ -37,6 +53,7 @@ sat_status fail(sat_status s, const char* fmt, ...);
 sat_status cuda_fail(cudaError_t e, const char* what);
 int getenv_int(const char* name, int dflt);
 int cluster_index(int cl);
+int default_cluster(int base_pair, int64_t bands);
 size_t in_size(sat_pair p);
 size_t out_size(sat_pair p);
 int tile_w(sat_pair p);

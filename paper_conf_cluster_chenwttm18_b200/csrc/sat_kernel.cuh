@@ -39,21 +39,30 @@
 //       the look-back warps (block partial-sum scan, Fig. 3c);
 //       the same scan over the cluster's CTAs runs in the leader.
 //
-// Warp roles (one CTA = 8 compute warps + 1 producer warp + kNLB look-back
-// warps):
+// Warp roles (one CTA = NCW compute warps + producer + aggregate + offset +
+// kNLW leader warps):
 //   producer : the leader's producer draws cluster tickets (atomic counter =>
 //              forward progress), late enough that a drawn band is active, and
 //              hands them to the cluster's other producers through DSMEM; each
 //              producer streams its band's tiles into an NSTAGE-deep smem ring
 //              with TMA (cp.async.bulk.tensor.3d + mbarrier complete_tx), or
 //              with plain loads on the generic (unaligned) path;
-//   compute  : pass A of chunk q (row + column scans -> the warp's column
-//              totals, row carries advanced), and, LOOK chunks later, pass B
-//              of chunk q: the same scans re-run from the still-resident smem
-//              tile plus the fix-up offset, stored straight to HBM;
-//   look-back: warp i handles chunks q = i (mod kNLB): band aggregate -> leader,
-//              (leader: cluster scan + global look-back + V_up to every band),
-//              per-warp fix-up offsets.
+//   aggregate: as soon as a tile lands, computes the band's vertical aggregate
+//              for that chunk straight from the input -- the column totals of
+//              R over the band's rows = (band input left of the chunk) + the
+//              prefix over x of the tile's column sums -- and sends it to the
+//              chunk's leader CTA.  Aggregates thus leave NSTAGE + LOOK + 1
+//              chunks ahead of the stores that need the carries, so the
+//              cross-cluster look-back mostly finds published predecessors;
+//   compute  : pass A of chunk q (row + column scans -> TMEM S' and the warp's
+//              column totals, row carries advanced), and, LOOK chunks later,
+//              pass B of chunk q: S' back from TMEM plus the fix-up offset,
+//              stored straight to HBM;
+//   offset   : the block partial-sum scan over the compute warps' column totals
+//               -> per-warp fix-up offsets;
+//   leader   : for the chunks this CTA leads (q = rank mod CL): segmented scan
+//              of the cluster's aggregates, global look-back, publication of
+//              the cluster's inclusive prefix, V_up to every band of the cluster.
 #pragma once
 
 #include <cuda.h>
@@ -70,10 +79,10 @@ constexpr int kShort = 5;
 template <int P>
 constexpr int kBase = P % kShort;
 
-#ifndef SAT_NLB
-#define SAT_NLB 3
+#ifndef SAT_NLW
+#define SAT_NLW 1
 #endif
-constexpr int kNLB = SAT_NLB;                    // look-back warps
+constexpr int kNLW = SAT_NLW;                    // leader (look-back) warps
 constexpr uint32_t kFull = 0xffffffffu;
 
 // Carry word tag (high 32 bits): (epoch << 2) | st,  st: 1 aggregate, 2 inclusive.
@@ -98,7 +107,7 @@ struct Cfg<P8U32S> {
   static constexpr int NCW = SAT_NCW8;   // compute warps, 4 rows each
   static constexpr int TH = 4 * NCW;     // 32 (2 CTAs per SM) or 64 (1 CTA per SM, 16 warps)
 #ifndef SAT_NST8
-#define SAT_NST8 4
+#define SAT_NST8 5
 #endif
   static constexpr int NSTAGE = SAT_NST8;  // TMA prefetch depth (stages free after pass A)
 };
@@ -164,15 +173,20 @@ template <>
 struct Cfg<P32S32S + kShort> : CfgShort<P32S32S> {};
 
 
-// Warp roles: NCW compute warps, then the producer, then kNLB look-back warps.
+// Warp roles: NCW compute warps, the producer, the aggregate warp, the offset
+// warp, then kNLW leader warps.
 template <int P>
 constexpr int kNCW = Cfg<P>::NCW;
 template <int P>
 constexpr int kProducerWarp = kNCW<P>;
 template <int P>
-constexpr int kFirstLbWarp = kNCW<P> + 1;
+constexpr int kAggWarp = kNCW<P> + 1;
 template <int P>
-constexpr int kThreads = (kNCW<P> + 1 + kNLB) * 32;
+constexpr int kOffWarp = kNCW<P> + 2;
+template <int P>
+constexpr int kFirstLwWarp = kNCW<P> + 3;
+template <int P>
+constexpr int kThreads = (kFirstLwWarp<P> + kNLW) * 32;
 
 // Words of one carry payload vector: TW elements * (4 / E) 64-bit words per element.
 template <int P>
@@ -180,13 +194,20 @@ constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
 // Payload vectors one look-back round lands in shared memory (kLandWords * 8 B
 // per look-back warp).
 #ifndef SAT_LAND_WORDS
-#define SAT_LAND_WORDS 512
+#define SAT_LAND_WORDS 256
 #endif
 template <int P>
-constexpr int kLandVecs = (SAT_LAND_WORDS) / kVecWords<P>;
+constexpr int kLandVecs = (SAT_LAND_WORDS) / kVecWords<P> > 2 ? (SAT_LAND_WORDS) / kVecWords<P> : 2;
 
+// Chunk slots between pass A and pass B (TMEM S', column totals, metadata).
 template <int P>
-constexpr int kNTot = (Cfg<P>::LOOK + 1 > kNLB) ? Cfg<P>::LOOK + 1 : kNLB;  // >= kNLB (phase safety)
+constexpr int kNTot = Cfg<P>::LOOK + 1;
+// V_up ring: the aggregate warp (which arms a slot) runs at most NSTAGE + kNTot
+// chunks ahead of pass B (which drains it): a stage is refilled only after
+// every compute warp's pass A of it, which follows that warp's pass B of the
+// chunk kNTot earlier.
+template <int P>
+constexpr int kNV = Cfg<P>::NSTAGE + kNTot<P>;
 
 // Tensor memory (TMEM) holds pass A's column-scanned rows S' until pass B:
 // per warp and chunk slot, RW rows x G x E values of 32-bit words (fp64: 2 words).
@@ -234,6 +255,11 @@ struct KParams {
   const uint64_t* chain_in;              // [nchunks][kVecWords] or NULL
   uint64_t* chain_out;                   // [nchunks][kVecWords] or NULL
   uint32_t chain_epoch;                  // >= 1; tag = (chain_epoch << 2) | kStIncl
+  // Bounded waits: a cross-CTA / cross-GPU carry wait that exceeds spin_ns
+  // sets bit 0 of *err, takes zeros and lets the launch finish (the host
+  // reports SAT_ERR_TIMEOUT) instead of hanging the GPU.
+  uint32_t* err;
+  uint64_t spin_ns;
 };
 
 // Optional phase profiling (debug builds with -DSAT_PROFILE): per-CTA shared
@@ -257,6 +283,11 @@ __device__ __forceinline__ uint64_t gtime() {
 #ifdef SAT_TIMELINE
 constexpr int kTlChunks = 256;
 __device__ unsigned long long g_sat_tl[1024][2 + kTlChunks];
+__device__ unsigned long long g_sat_tl_agg[1024][kTlChunks];  // aggregate sent (first band)
+__device__ unsigned long long g_sat_tl_v[1024][kTlChunks];    // V_up landed (first band)
+__device__ unsigned long long g_sat_tl_ls[1024][kTlChunks];   // leader: gather complete (led chunks)
+__device__ unsigned long long g_sat_tl_lt[1024][kTlChunks];   // leader: prefix known
+__device__ unsigned long long g_sat_tl_ld[1024][kTlChunks];   // leader: V_up sent
 __device__ __forceinline__ uint64_t tl_now() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -283,11 +314,17 @@ enum ProfSlot {
 };
 
 // Chunk q of a cluster is led by CTA q % CL (rotating leadership spreads the
-// global look-backs over all the cluster's look-back warps).  A leader's
-// gather slot is reused CL * kNLead chunks later, which must be >= kNTot so a
-// band cannot send a new aggregate into a slot its leader still reads.
+// global look-backs over all the cluster's leader warps).  A leader's gather
+// slot is reused CL * kNLead chunks later.  A band's aggregate warp reaches
+// chunk q only after the band's pass B of chunk q - NSTAGE - kNTot, i.e. after
+// that chunk's leader has read the band's earlier aggregate, so CL * kNLead >=
+// NSTAGE + kNTot keeps a slot from being overwritten while its leader reads it.
+// The end-of-work sentinels go up to CL * kNLW - 1 chunks further (the next
+// chunk each leader warp would lead), hence the extra CL * kNLW - 1.
 template <int P, int CL>
-constexpr int kNLead = (kNTot<P> + CL - 1) / CL;
+constexpr int kNLeadRaw = (Cfg<P>::NSTAGE + kNTot<P> + CL * kNLW - 1 + CL - 1) / CL;
+template <int P, int CL>
+constexpr int kNLead = kNLeadRaw<P, CL> > kNLW ? kNLeadRaw<P, CL> : kNLW;
 
 template <int P, int CL>
 struct __align__(128) Smem {
@@ -295,17 +332,19 @@ struct __align__(128) Smem {
   typename C::TA in[C::NSTAGE][C::TH][C::TW];   // TMA destination ring
   alignas(128) typename C::TB tot[kNTot<P>][kNCW<P>][C::TW];    // per-warp column totals -> fix-up offsets
   alignas(128) typename C::TB lead_in[kNLead<P, CL>][CL][C::TW];  // chunk leader: the bands' aggregates
-  alignas(128) typename C::TB vin[kNTot<P>][C::TW];          // V_up of this band (from the leader)
+  alignas(128) typename C::TB vin[kNV<P>][C::TW];            // V_up of this band (from the leader)
   int32_t meta[kNCW<P>][kNTot<P>][4];              // per warp: (band lo, img, k, chunk) of each slot
   uint32_t tmem_base;                           // TMEM address from tcgen05.alloc
-  alignas(128) uint64_t land[kNLB][kLandVecs<P>][kVecWords<P>];  // look-back payload landing (bulk copies)
+  alignas(128) uint64_t land[kNLW][kLandVecs<P>][kVecWords<P>];  // look-back landing (bulk copies)
   uint64_t full[C::NSTAGE];
   uint64_t empty[C::NSTAGE];
   uint64_t tot_full[kNTot<P>];
   uint64_t carry_full[kNTot<P>];
-  uint64_t lead_full[kNLead<P, CL>];            // tx: CL aggregates landed in lead_in
-  uint64_t vin_full[kNTot<P>];                  // tx: V_up landed in vin
-  uint64_t land_full[kNLB];                     // tx: a look-back round landed
+  uint64_t lead_full[kNLead<P, CL>];            // CL aggregates landed in lead_in (+ leader's arrive)
+  int64_t lead_band[kNLead<P, CL>];             // leader: its own band of the slot's chunk (-1: end)
+  int32_t lead_chunk[kNLead<P, CL>];
+  uint64_t vin_full[kNV<P>];                    // tx: V_up landed in vin
+  uint64_t land_full[kNLW];                     // tx: a look-back round landed
   uint64_t tk_full;                             // tx: ticket landed in tk_slot
   uint64_t tk_empty;                            // leader: peers consumed the ticket
   int64_t tk_slot;
@@ -848,6 +887,17 @@ __device__ __forceinline__ uint64_t* payload_row(const KParams& p, int64_t T, in
   return reinterpret_cast<uint64_t*>(p.payload) + ((T * p.nchunks + chunk) * (int64_t)kVecWords<P>);
 }
 
+__device__ __forceinline__ uint64_t gclock() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// A bounded wait ran out: flag it (the host turns it into SAT_ERR_TIMEOUT).
+__device__ __forceinline__ void flag_timeout(const KParams& p) {
+  if (p.err) atomicOr(p.err, 1u);
+}
+
 // Status-tagged words: high 32 bits = (epoch << 2) | st, st = kStAgg or kStIncl.
 // One vector per (cluster ticket, chunk): written first as the aggregate, then
 // overwritten in place by the inclusive prefix.  A reader classifies a vector
@@ -869,12 +919,11 @@ __device__ __forceinline__ void debug_delay(uint32_t salt) {
 #endif
 
 template <int P>
-__device__ __forceinline__ void publish(const KParams& p, int64_t T, int32_t chunk, uint32_t st,
+__device__ __forceinline__ void publish(const KParams& p, uint64_t* row, uint32_t st,
                                         const typename Cfg<P>::TB (&v)[Cfg<P>::G][Cfg<P>::E],
                                         int lane) {
   using C = Cfg<P>;
-  SAT_DELAY(st + 17u * chunk);
-  uint64_t* row = payload_row<P>(p, T, chunk);
+  SAT_DELAY(st + 17u * (uint32_t)(uintptr_t)row);
 #pragma unroll
   for (int g = 0; g < C::G; ++g) {
     uint64_t w[4];
@@ -896,9 +945,9 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
-// Decoupled look-back up the tile column over cluster tickets: V = sum of the
-// predecessors' aggregates down to (and including) the nearest inclusive
-// prefix.  Each round lands up to kLandVecs predecessor vectors in shared
+// Decoupled look-back up the tile column over cluster tickets:
+// V = sum of the predecessors' aggregates down to (and including) the nearest
+// inclusive prefix.  Each round lands up to kLandVecs predecessor vectors in shared
 // memory with bulk copies (one per vector, on the TMA engine): one L2 round
 // trip per round, no separate status probe.  Vectors are classified by warp
 // votes on the word tags (each lane checks its own words).
@@ -918,6 +967,7 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
 #pragma unroll
     for (int e = 0; e < C::E; ++e) V[g][e] = TB(0);
   int64_t j = T - 1;
+  uint64_t t_start = 0;
   for (;;) {
     const int nb = (j - first + 1) < B ? (int)(j - first + 1) : B;
     int kk = nb;  // index of the inclusive vector in this round (nb: none)
@@ -960,6 +1010,11 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
       }
       if (ready) break;
       SAT_PADD(sm, kPfLbRetries, 1);
+      if (t_start == 0) t_start = gclock();
+      if (gclock() - t_start > p.spin_ns) {  // bounded wait: flag, go on with what is summed
+        if (lane == 0) flag_timeout(p);
+        return;
+      }
       __nanosleep(32);
     }
     const int nsum = kk < nb ? kk + 1 : nb;
@@ -1012,6 +1067,7 @@ __device__ __forceinline__ void chain_wait(const KParams& p, int32_t chunk,
   using C = Cfg<P>;
   const uint64_t* row = p.chain_in + (int64_t)chunk * kVecWords<P>;
   const uint32_t want = (p.chain_epoch << 2) | kStIncl;
+  const uint64_t t_start = gclock();
   for (;;) {
     bool ok = true;
     uint64_t w[C::G][4];
@@ -1026,6 +1082,14 @@ __device__ __forceinline__ void chain_wait(const KParams& p, int32_t chunk,
     if (__all_sync(kFull, ok)) {
 #pragma unroll
       for (int g = 0; g < C::G; ++g) Tag<kBase<P>>::dec(w[g], V[g]);
+      return;
+    }
+    if (gclock() - t_start > p.spin_ns) {  // the band above never published: zeros, flag
+      if (lane == 0) flag_timeout(p);
+#pragma unroll
+      for (int g = 0; g < C::G; ++g)
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) V[g][e] = typename C::TB(0);
       return;
     }
     __nanosleep(64);
@@ -1048,22 +1112,18 @@ __device__ __forceinline__ void load_carry_in(const KParams& p, int32_t chunk,
     }
 }
 
-// Leader CTA, chunk q (slot t): wait for the cluster's CL band aggregates,
-// publish / look back for the cluster, and send every band of the cluster its
-// V_up (segmented at image starts inside the cluster).
+// Leader CTA, chunk q (V_up slot v, gather slot ls, whose CL band aggregates
+// have landed): publish / look back for the cluster, publish its inclusive
+// prefix, and send every band of the cluster its V_up (segmented at image
+// starts inside the cluster).
 template <int P, int CL>
 __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, int lbw,
-                                             uint32_t& land_ph, int t, int ls, uint32_t lph,
-                                             int64_t g0, int32_t chunk, int lane) {
+                                             uint32_t& land_ph, int v, int ls, int64_t g0,
+                                             int32_t chunk, uint32_t qdbg, int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
-  constexpr uint32_t kVecBytes = C::TW * sizeof(TB);
   const int32_t n0 = (int32_t)(g0 / p.bands_per_image);
   const int32_t k0 = (int32_t)(g0 - (int64_t)n0 * p.bands_per_image);
-  SAT_PT(t0);
-  mbar_wait_cluster(&sm.lead_full[ls], lph);
-  SAT_PT(t1);
-  SAT_PADD(sm, kPfLbCluster, t1 - t0);
   SAT_PADD(sm, kPfLeaderChunks, 1);
   const int64_t T = g0 / CL;
   const int64_t bpi = p.bands_per_image;
@@ -1104,18 +1164,16 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
     chain_wait<P>(p, chunk, carry0, lane);  // the band above publishes it chunk by chunk
   else
     load_carry_in<P>(p, chunk, carry0, lane);
-  if (has_succ) {
-    if (tail_self) {
-      TB incl[C::G][C::E];
+  // The cluster's contribution to its tail image goes out first -- the clusters
+  // below need it -- then, as a reader of its head image, the look-back.
+  TB contrib[C::G][C::E];
 #pragma unroll
-      for (int g = 0; g < C::G; ++g)
+  for (int g = 0; g < C::G; ++g)
 #pragma unroll
-        for (int e = 0; e < C::E; ++e) incl[g][e] = carry0[g][e] + tail[g][e];
-      publish<P>(p, T, chunk, kStIncl, incl, lane);
-    } else {
-      publish<P>(p, T, chunk, kStAgg, tail, lane);
-    }
-  }
+    for (int e = 0; e < C::E; ++e) contrib[g][e] = tail_self ? carry0[g][e] + tail[g][e] : tail[g][e];
+  // aggregate, or -- when the tail segment starts its image -- already inclusive
+  if (has_succ)
+    publish<P>(p, payload_row<P>(p, T, chunk), tail_self ? kStIncl : kStAgg, contrib, lane);
   TB Vcl[C::G][C::E];
 #ifdef SAT_DEBUG_NO_LOOKBACK  // timing experiments only: wrong results, no cross-cluster wait
 #pragma unroll
@@ -1127,11 +1185,22 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
   if (!head_self) {
 #endif
     SAT_PT(t2);
-    const int64_t first = ((int64_t)n0 * bpi) / CL;
-    lookback<P>(sm, sm.land[lbw], &sm.land_full[lbw], land_ph, p, T, first, chunk, Vcl, lane);
+    const int64_t T0 = ((int64_t)n0 * bpi) / CL;  // first cluster of the head image
+    lookback<P>(sm, sm.land[lbw], &sm.land_full[lbw], land_ph, p, T, T0, chunk, Vcl, lane);
+    if (has_succ && !tail_self) {  // the cluster's inclusive prefix (overwrites its aggregate)
+      TB incl[C::G][C::E];
+#pragma unroll
+      for (int g = 0; g < C::G; ++g)
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) incl[g][e] = Vcl[g][e] + tail[g][e];
+      publish<P>(p, payload_row<P>(p, T, chunk), kStIncl, incl, lane);
+    }
     SAT_PT(t3);
     SAT_PADD(sm, kPfLbLookback, t3 - t2);
   }
+#ifdef SAT_TIMELINE
+  if (lane == 0 && blockIdx.x < 1024 && qdbg < kTlChunks) g_sat_tl_lt[blockIdx.x][qdbg] = tl_now();
+#endif
   // Pass 2: V_up of every band of the cluster (padding CTAs get zeros).
   {
     const uint32_t self = CL > 1 ? cluster_rank() : 0u;
@@ -1151,99 +1220,315 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
       }
 #pragma unroll
       for (int g = 0; g < C::G; ++g) {
-        TB v[C::E], a[C::E];
+        TB vv[C::E], a[C::E];
         // read this band's aggregate BEFORE sending it its V_up: once CTA r has
         // its V_up it may eventually overwrite lead_in[ls][r] for a later chunk
         unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.lead_in[ls][r][col_of<P>(g, lane)]),
                            a);
 #pragma unroll
         for (int e = 0; e < C::E; ++e) {
-          v[e] = valid ? run[g][e] : TB(0);
+          vv[e] = valid ? run[g][e] : TB(0);
           if (valid) run[g][e] += a[e];
         }
-        send16(&sm.vin[t][col_of<P>(g, lane)], &sm.vin_full[t], (uint32_t)r, self, pack16<TB, C::E>(v));
+        send16(&sm.vin[v][col_of<P>(g, lane)], &sm.vin_full[v], (uint32_t)r, self, pack16<TB, C::E>(vv));
       }
       if ((uint32_t)r == self) {
         __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.vin_full[t]);
+        if (lane == 0) mbar_arrive(&sm.vin_full[v]);
       }
       if (++k == bpi) k = 0;
     }
     // The image's bottom row S(r1-1, .) = the tail segment's inclusive value.
     if (!has_succ && p.chain_out != nullptr) chain_publish<P>(p, chunk, run, lane);
   }
-  if (has_succ && !tail_self) {
-    TB incl[C::G][C::E];
-#pragma unroll
-    for (int g = 0; g < C::G; ++g)
-#pragma unroll
-      for (int e = 0; e < C::E; ++e) incl[g][e] = Vcl[g][e] + tail[g][e];
-    publish<P>(p, T, chunk, kStIncl, incl, lane);
-  }
-  (void)kVecBytes;
 }
 
-template <int P, int CL>
-__device__ __forceinline__ void lookback_warp(Smem<P, CL>& sm, const KParams& p, int lbw,
-                                              uint32_t rank, int lane) {
+template <typename TB>
+__device__ __forceinline__ TB from_bits(uint64_t b) {
+  TB v;
+  memcpy(&v, &b, sizeof(TB));
+  return v;
+}
+
+// Offset step (chunk q, its column totals and V_up landed): block partial-sum
+// scan (Fig. 3c) over the compute warps' column totals, started
+// from the band's V_up (and the exclusive layout's nVal) -> each compute
+// warp's complete fix-up offset, in place.  One warp per CTA waits for V_up
+// (cluster-scope acquire); the compute warps wait only for its local arrival.
+template <int P, int CL, bool kEx>
+__device__ __forceinline__ void offset_step(Smem<P, CL>& sm, const KParams& p, uint32_t q,
+                                            int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
-  constexpr int NT = kNTot<P>;
-  constexpr uint32_t kVecBytes = C::TW * sizeof(TB);
+  const int t = q % kNTot<P>;
+  const int vs = q % kNV<P>;
+#ifdef SAT_TIMELINE
+  if (lane == 0 && blockIdx.x < 1024 && q < kTlChunks) g_sat_tl_v[blockIdx.x][q] = tl_now();
+#endif
+#pragma unroll
+  for (int g = 0; g < C::G; ++g) {
+    TB run[C::E];
+    unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.vin[vs][col_of<P>(g, lane)]), run);
+    if constexpr (kEx) {
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) run[e] += from_bits<TB>(p.nval_bits);
+    }
+#pragma unroll
+    for (int w = 0; w < kNCW<P>; ++w) {
+      uint4* cell = reinterpret_cast<uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]);
+      TB tt[C::E];
+      unpack16<TB, C::E>(*cell, tt);
+      *cell = pack16<TB, C::E>(run);
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) run[e] += tt[e];
+    }
+  }
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&sm.carry_full[t]);
+}
+
+// Leader warp lw: the chunks this CTA leads, q = rank + CL * j for
+// j = lw (mod kNLW), each as soon as the cluster's aggregates have landed.
+template <int P, int CL>
+__device__ __forceinline__ void leader_warp(Smem<P, CL>& sm, const KParams& p, int lw,
+                                            uint32_t rank, int lane) {
   uint32_t land_ph = 0;
-  for (uint32_t q = lbw;; q += kNLB) {
-    const int t = q % NT;
+  for (uint32_t j = lw;; j += kNLW) {
+    const int ls = j % kNLead<P, CL>;
     SAT_PT(t0);
-    mbar_wait(&sm.tot_full[t], (q / NT) & 1);
+    mbar_wait_cluster(&sm.lead_full[ls], (j / kNLead<P, CL>) & 1);
     SAT_PT(t1);
-    SAT_PADD(sm, kPfLbWaitTot, t1 - t0);
-    const int64_t band = sm.tot_band[t];
+    SAT_PADD(sm, kPfLbCluster, t1 - t0);
+    const int64_t band = sm.lead_band[ls];
     if (band < 0) break;
     SAT_PADD(sm, kPfLbChunks, 1);
-    const int32_t chunk = sm.tot_chunk[t];
-    // Chunk q is led by CTA q % CL; its gather slot and that slot's phase.
-    const uint32_t lead = q % CL;
-    const uint32_t m = q / CL;
-    const int ls = m % kNLead<P, CL>;
-    const uint32_t lph = (m / kNLead<P, CL>) & 1;
-    SAT_DELAY(7u * q + rank);
-    // Arm the V_up receive before our aggregate can reach the leader.  The
-    // leader's own hand-offs are shared stores + arrive (see send16), so it
-    // arms only the bytes of its CL-1 peers.
+    const uint32_t q = rank + CL * j;
+#ifdef SAT_TIMELINE
+    if (lane == 0 && blockIdx.x < 1024 && q < kTlChunks) g_sat_tl_ls[blockIdx.x][q] = tl_now();
+#endif
+    leader_chunk<P, CL>(sm, p, lw, land_ph, (int)(q % kNV<P>), ls, band - rank, sm.lead_chunk[ls],
+                        q, lane);
+#ifdef SAT_TIMELINE
+    if (lane == 0 && blockIdx.x < 1024 && q < kTlChunks) g_sat_tl_ld[blockIdx.x][q] = tl_now();
+#endif
+  }
+  // the last node stores must have read their staging buffer before the CTA exits
+  if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  __syncwarp();
+}
+
+// Aggregate warp helpers: the band's vertical aggregate of a landed tile,
+//   agg(x) = L + sum_{x0 <= x' <= x} colsum(x'),  colsum(x') = sum_{y in band} A(y, x'),
+// L = the band's input left of the chunk (= sum_y rowcarry(y)); this equals
+// sum_y R(y, x), the column total of the row-prefixed values (Sec. 5).
+// 8u: column sums of bytes in packed 16-bit lanes (<= TH * 255 < 2^16), then
+// the in-lane prefix and a Kogge-Stone scan of the lane totals (Alg. 2, 3).
+template <int TH>
+__device__ __forceinline__ void colsum8(const uint8_t* tile, int lane, uint32_t (&c)[2][4]) {
+  uint32_t lo[2] = {0u, 0u}, hi[2] = {0u, 0u};
+#pragma unroll 8
+  for (int r = 0; r < TH; ++r) {
+#pragma unroll
+    for (int g = 0; g < 2; ++g) {
+      const uint32_t w = *reinterpret_cast<const uint32_t*>(tile + r * 256 + g * 128 + 4 * lane);
+      lo[g] += __byte_perm(w, 0u, 0x4240);  // bytes 0, 2 -> 16-bit lanes
+      hi[g] += __byte_perm(w, 0u, 0x4341);  // bytes 1, 3
+    }
+  }
+#pragma unroll
+  for (int g = 0; g < 2; ++g) {
+    c[g][0] = lo[g] & 0xFFFFu;
+    c[g][1] = hi[g] & 0xFFFFu;
+    c[g][2] = lo[g] >> 16;
+    c[g][3] = hi[g] >> 16;
+  }
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_incl(T v, int lane) {
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const T o = __shfl_up_sync(kFull, v, d);
+    if (lane >= d) v += o;
+  }
+  return v;
+}
+
+// Per-pair aggregate of one tile; `L` is the running band-left sum (reset at chunk 0).
+template <int P>
+struct Agg;
+template <>
+struct Agg<P8U32S> {
+  using Acc = uint32_t;
+  template <int TH>
+  static __device__ __forceinline__ void run(const uint8_t* tile, int lane, Acc& L,
+                                             uint32_t (&agg)[2][4]) {
+    uint32_t c[2][4];
+    colsum8<TH>(tile, lane, c);
+    uint32_t pg[2][4], inc[2];
+#pragma unroll
+    for (int g = 0; g < 2; ++g) {
+      pg[g][0] = c[g][0];
+#pragma unroll
+      for (int e = 1; e < 4; ++e) pg[g][e] = pg[g][e - 1] + c[g][e];
+      inc[g] = warp_incl(pg[g][3], lane);
+    }
+    const uint32_t tot0 = __shfl_sync(kFull, inc[0], 31), tot1 = __shfl_sync(kFull, inc[1], 31);
+    const uint32_t b0 = L + (inc[0] - pg[0][3]), b1 = L + tot0 + (inc[1] - pg[1][3]);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      agg[0][e] = b0 + pg[0][e];
+      agg[1][e] = b1 + pg[1][e];
+    }
+    L += tot0 + tot1;
+  }
+};
+template <>
+struct Agg<P8U32F> {
+  using Acc = uint64_t;  // exact integer sums, rounded once to fp32
+  template <int TH>
+  static __device__ __forceinline__ void run(const uint8_t* tile, int lane, Acc& L,
+                                             float (&agg)[2][4]) {
+    uint32_t c[2][4];
+    colsum8<TH>(tile, lane, c);
+    uint32_t pg[2][4], inc[2];
+#pragma unroll
+    for (int g = 0; g < 2; ++g) {
+      pg[g][0] = c[g][0];
+#pragma unroll
+      for (int e = 1; e < 4; ++e) pg[g][e] = pg[g][e - 1] + c[g][e];
+      inc[g] = warp_incl(pg[g][3], lane);
+    }
+    const uint32_t tot0 = __shfl_sync(kFull, inc[0], 31), tot1 = __shfl_sync(kFull, inc[1], 31);
+    const uint32_t b0 = inc[0] - pg[0][3], b1 = tot0 + (inc[1] - pg[1][3]);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      agg[0][e] = (float)(L + (uint64_t)(b0 + pg[0][e]));
+      agg[1][e] = (float)(L + (uint64_t)(b1 + pg[1][e]));
+    }
+    L += (uint64_t)tot0 + tot1;
+  }
+};
+template <typename T>
+struct AggWide {  // 4-byte elements, 128-column tiles: lane owns columns 4l .. 4l+3
+  using Acc = T;
+  template <int TH>
+  static __device__ __forceinline__ void run(const T* tile, int lane, Acc& L, T (&agg)[1][4]) {
+    T c[4] = {T(0), T(0), T(0), T(0)};
+#pragma unroll 8
+    for (int r = 0; r < TH; ++r) {
+      const uint4 w = *reinterpret_cast<const uint4*>(tile + r * 128 + 4 * lane);
+      T a[4];
+      unpack16<T, 4>(w, a);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) c[e] += a[e];
+    }
+    T pg[4];
+    pg[0] = c[0];
+#pragma unroll
+    for (int e = 1; e < 4; ++e) pg[e] = pg[e - 1] + c[e];
+    const T inc = warp_incl(pg[3], lane);
+    const T tot = __shfl_sync(kFull, inc, 31);
+    T ex = __shfl_up_sync(kFull, inc, 1);
+    if (lane == 0) ex = T(0);
+    const T b = L + ex;
+#pragma unroll
+    for (int e = 0; e < 4; ++e) agg[0][e] = b + pg[e];
+    L += tot;
+  }
+};
+template <>
+struct Agg<P32F32F> : AggWide<float> {};
+template <>
+struct Agg<P32S32S> : AggWide<uint32_t> {};
+template <>
+struct Agg<P64F64F> {
+  using Acc = double;
+  template <int TH>
+  static __device__ __forceinline__ void run(const double* tile, int lane, Acc& L,
+                                             double (&agg)[1][2]) {
+    double c0 = 0.0, c1 = 0.0;
+#pragma unroll 8
+    for (int r = 0; r < TH; ++r) {
+      const double2 a = *reinterpret_cast<const double2*>(tile + r * 64 + 2 * lane);
+      c0 += a.x;
+      c1 += a.y;
+    }
+    const double p1 = c0 + c1;
+    const double inc = warp_incl(p1, lane);
+    const double tot = __shfl_sync(kFull, inc, 31);
+    double ex = __shfl_up_sync(kFull, inc, 1);
+    if (lane == 0) ex = 0.0;
+    const double b = L + ex;
+    agg[0][0] = b + c0;
+    agg[0][1] = b + p1;
+    L += tot;
+  }
+};
+
+// Aggregate step (stage of chunk q landed): the band aggregate of the tile ->
+// the chunk's leader.  Returns false at the end-of-work sentinel, after giving
+// every leader warp of this CTA a sentinel in the gather slot of the next
+// chunk it would lead (its peers send nothing there).
+template <int P, int CL>
+__device__ __forceinline__ bool aggregate_step(Smem<P, CL>& sm, uint32_t rank, uint32_t q,
+                                               typename Agg<kBase<P>>::Acc& L, int lane) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  using A = Agg<kBase<P>>;
+  constexpr uint32_t kVecBytes = C::TW * sizeof(TB);
+  const int s = q % C::NSTAGE;
+  const int64_t band = sm.stage_band[s];
+  const uint32_t lead = q % CL;
+  if (band < 0) {
     if (lane == 0) {
-      if (rank != lead) {
-        mbar_arrive_expect_tx(&sm.vin_full[t], kVecBytes);
-      } else if (CL > 1) {
-        mbar_expect_tx(&sm.lead_full[ls], (CL - 1) * kVecBytes);
+      const uint32_t jn = q <= rank ? 0u : (q - rank + CL - 1) / CL;
+      for (int i = 0; i < kNLW; ++i) {
+        const uint32_t j = jn + (uint32_t)(((i - (int)(jn % kNLW)) % kNLW + kNLW) % kNLW);
+        const int ls = j % kNLead<P, CL>;
+        sm.lead_band[ls] = -1;
+        mbar_arrive(&sm.lead_full[ls]);
       }
     }
-    TB agg[C::G][C::E];
-#pragma unroll
-    for (int g = 0; g < C::G; ++g) {
-#pragma unroll
-      for (int e = 0; e < C::E; ++e) agg[g][e] = TB(0);
-#pragma unroll
-      for (int w = 0; w < kNCW<P>; ++w) {
-        uint4* cell = reinterpret_cast<uint4*>(&sm.tot[t][w][col_of<P>(g, lane)]);
-        TB tt[C::E];
-        unpack16<TB, C::E>(*cell, tt);
-        *cell = pack16<TB, C::E>(agg[g]);
-#pragma unroll
-        for (int e = 0; e < C::E; ++e) agg[g][e] += tt[e];
-      }
-    }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&sm.carry_full[t]);
+    return false;
+  }
+  const int32_t chunk = sm.stage_chunk[s];
+  TB agg[C::G][C::E];
+  if (chunk == 0) L = typename A::Acc(0);
+  A::template run<C::TH>(&sm.in[s][0][0], lane, L, agg);
+  if (sm.stage_img[s] < 0) {  // padding band of a partial cluster: stage not loaded
 #pragma unroll
     for (int g = 0; g < C::G; ++g)
-      send16(&sm.lead_in[ls][rank][col_of<P>(g, lane)], &sm.lead_full[ls], lead, rank,
-             pack16<TB, C::E>(agg[g]));
-    if (lead == rank) {  // own contribution went by shared stores
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&sm.lead_full[ls]);
-    }
-    if (rank == lead) leader_chunk<P, CL>(sm, p, lbw, land_ph, t, ls, lph, band - rank, chunk, lane);
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) agg[g][e] = TB(0);
   }
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&sm.empty[s]);
+  const int ls = (q / CL) % kNLead<P, CL>;
+  // Arm the V_up receive before our aggregate can reach the leader.  The
+  // leader's own hand-offs are shared stores + arrive (see send16), so it
+  // arms only the bytes of its CL-1 peers.
+  if (lane == 0) {
+    if (rank != lead) {
+      mbar_arrive_expect_tx(&sm.vin_full[q % kNV<P>], kVecBytes);
+    } else {
+      if (CL > 1) mbar_expect_tx(&sm.lead_full[ls], (CL - 1) * kVecBytes);
+      sm.lead_band[ls] = band;
+      sm.lead_chunk[ls] = chunk;
+    }
+  }
+#pragma unroll
+  for (int g = 0; g < C::G; ++g)
+    send16(&sm.lead_in[ls][rank][col_of<P>(g, lane)], &sm.lead_full[ls], lead, rank,
+           pack16<TB, C::E>(agg[g]));
+  if (lead == rank) {  // own contribution went by shared stores
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sm.lead_full[ls]);
+  }
+#ifdef SAT_TIMELINE
+  if (lane == 0 && blockIdx.x < 1024 && q < kTlChunks) g_sat_tl_agg[blockIdx.x][q] = tl_now();
+#endif
+  return true;
 }
 
 // ---------------------------------------------------------------------------
@@ -1326,12 +1611,6 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint3
 
 // Pass B of chunk q: wait for the fix-up offsets, load S' back from TMEM,
 // add, store (a8).
-template <typename TB>
-__device__ __forceinline__ TB from_bits(uint64_t b) {
-  TB v;
-  memcpy(&v, &b, sizeof(TB));
-  return v;
-}
 
 // Exclusive-layout store of one tile row (Eq. 2; NPP layout):
 // S(y, x) goes to output column o = x + 1.  The 16-B aligned output vector of
@@ -1382,27 +1661,17 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   const int t = q % kNTot<P>;
   SAT_PT(t0);
   mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
-  mbar_wait_cluster(&sm.vin_full[t], (q / kNTot<P>) & 1);
   SAT_PT(t1);
   if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
   const int32_t img = sm.meta[warp][t][1];
   if (img >= 0) {
     uint32_t w[NW];
     tmem_ld(tmem_addr(sm, t, warp), w);
-    TB off[C::G][C::E];
+    TB off[C::G][C::E];  // V_up + the warps above + nVal (offset warp)
 #pragma unroll
-    for (int g = 0; g < C::G; ++g) {
-      TB v[C::E];
+    for (int g = 0; g < C::G; ++g)
       unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.tot[t][warp][col_of<P>(g, lane)]),
                          off[g]);
-      unpack16<TB, C::E>(*reinterpret_cast<const uint4*>(&sm.vin[t][col_of<P>(g, lane)]), v);
-#pragma unroll
-      for (int e = 0; e < C::E; ++e) off[g][e] += v[e];
-      if constexpr (kEx) {
-#pragma unroll
-        for (int e = 0; e < C::E; ++e) off[g][e] += from_bits<TB>(p.nval_bits);
-      }
-    }
     const int64_t k = sm.meta[warp][t][2];
     const int32_t chunk = sm.meta[warp][t][3];
     const int64_t y0 = k * C::TH + warp * RW;
@@ -1500,10 +1769,9 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
       break;
     }
   }
-  // One end-of-work sentinel per look-back warp (slots are free: all pass B done).
-  for (int i = 0; i < kNLB; ++i) {
-    const uint32_t q = qa + i;
-    const int t = q % kNTot<P>;
+  // End-of-work sentinel for the offset warp (the slot is free: all pass B done).
+  {
+    const int t = qa % kNTot<P>;
     if (warp == 0 && lane == 0) sm.tot_band[t] = -1;
     __syncwarp();
     if (lane == 0) mbar_arrive(&sm.tot_full[t]);
@@ -1625,15 +1893,15 @@ __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
   if (threadIdx.x == 0) {
     for (int s = 0; s < C::NSTAGE; ++s) {
       mbar_init(&sm.full[s], 1);
-      mbar_init(&sm.empty[s], kNCW<P>);
+      mbar_init(&sm.empty[s], kNCW<P> + 1);  // compute warps' pass A + the aggregate warp
     }
     for (int t = 0; t < kNTot<P>; ++t) {
       mbar_init(&sm.tot_full[t], kNCW<P>);
       mbar_init(&sm.carry_full[t], 1);
-      mbar_init(&sm.vin_full[t], 1);
     }
+    for (int v = 0; v < kNV<P>; ++v) mbar_init(&sm.vin_full[v], 1);
     for (int i = 0; i < kNLead<P, CL>; ++i) mbar_init(&sm.lead_full[i], 1);
-    for (int i = 0; i < kNLB; ++i) mbar_init(&sm.land_full[i], 1);
+    for (int i = 0; i < kNLW; ++i) mbar_init(&sm.land_full[i], 1);
     mbar_init(&sm.tk_full, 1);
     mbar_init(&sm.tk_empty, CL > 1 ? CL - 1 : 1);
     sm.passA_done = 0;
@@ -1664,8 +1932,21 @@ __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
 #endif
   if (warp == kProducerWarp<P>) {
     producer_warp<P, CL, kTMA>(sm, p, &map, rank, lane);
-  } else if (warp >= kFirstLbWarp<P>) {
-    lookback_warp<P, CL>(sm, p, warp - kFirstLbWarp<P>, rank, lane);
+  } else if (warp == kAggWarp<P>) {
+    typename Agg<kBase<P>>::Acc L = typename Agg<kBase<P>>::Acc(0);
+    for (uint32_t q = 0;; ++q) {
+      mbar_wait(&sm.full[q % Cfg<P>::NSTAGE], (q / Cfg<P>::NSTAGE) & 1);
+      if (!aggregate_step<P, CL>(sm, rank, q, L, lane)) break;
+    }
+  } else if (warp == kOffWarp<P>) {
+    for (uint32_t q = 0;; ++q) {
+      mbar_wait(&sm.tot_full[q % kNTot<P>], (q / kNTot<P>) & 1);
+      if (sm.tot_band[q % kNTot<P>] < 0) break;
+      mbar_wait_cluster(&sm.vin_full[q % kNV<P>], (q / kNV<P>) & 1);
+      offset_step<P, CL, kEx>(sm, p, q, lane);
+    }
+  } else if (warp >= kFirstLwWarp<P>) {
+    leader_warp<P, CL>(sm, p, warp - kFirstLwWarp<P>, rank, lane);
   } else {
     compute_warp<P, CL, kVecOut, kEx>(sm, p, warp, lane);
   }

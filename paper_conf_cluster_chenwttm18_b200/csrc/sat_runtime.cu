@@ -89,7 +89,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
                            const ChainSpec* chain) {
   using C = Cfg<P>;
   const bool tma = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
-                   getenv_int("SAT_FORCE_GENERIC", 0) == 0;
+                   pl->force_generic == 0;
   const bool vec = ((uintptr_t)out % 16 == 0) && (op % 16 == 0) && (batch == 1 || ois % 16 == 0);
   KParams kp;
   kp.in = static_cast<const char*>(in);
@@ -109,9 +109,6 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.chain_in = chain ? static_cast<const uint64_t*>(chain->in) : nullptr;
   kp.chain_out = chain ? static_cast<uint64_t*>(chain->out) : nullptr;
   kp.chain_epoch = chain ? chain->epoch : 0;
-  if ((kp.total_bands + (P >= kShort ? 1 : 0)) / (P >= kShort ? 2 : 1) * kp.nchunks > pl->max_tiles)
-    return fail(SAT_ERR_INVALID_ARGUMENT, "problem needs %lld tiles, plan holds %lld",
-                (long long)(kp.total_bands * kp.nchunks), (long long)pl->max_tiles);
 
   CUtensorMap map;
   memset(&map, 0, sizeof(map));
@@ -133,6 +130,26 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
     if (r != CUDA_SUCCESS) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
   }
 
+  // Cluster size: 8 bands per cluster for the float pairs when there are enough
+  // bands to fill the machine (shorter look-back chains pay off there); 4 for
+  // 8u->32s and for short/wide images (measured, DESIGN.md Sec. 6).
+  int CL = default_cluster(kBase<P>, kp.total_bands);
+  if (pl->cluster > 0) CL = pl->cluster;
+  if (ex && CL != 4 && CL != 8) CL = 4;  // exclusive kernels: clusters of 4 and 8
+  if (P >= kShort) CL = 4;               // short-band kernels: clusters of 4 only
+  kp.total_tickets = (kp.total_bands + CL - 1) / CL;
+  // Look-back workspace: one tagged carry vector per (cluster ticket, chunk).
+  {
+    const size_t need = (size_t)kp.total_tickets * kp.nchunks * kVecWords<P> * 8;
+    const size_t have = pl->ws_bytes - ((char*)pl->payload - (char*)pl->ws);
+    if (need > have)
+      return fail(SAT_ERR_INVALID_ARGUMENT,
+                  "problem needs %zu bytes of carry workspace (cluster %d), plan holds %zu", need, CL,
+                  have);
+  }
+  kp.err = pl->err;
+  kp.spin_ns = pl->spin_ns;
+
   // Epoch: status words from earlier launches carry older epochs.
   if (pl->epoch + 1 >= (1u << 30)) {
     // status words hold 30 epoch bits and payload words 32: clear both on wrap
@@ -147,26 +164,12 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.ticket_base = pl->ticket_base;
 
   const int mode = (tma ? 1 : 0) | (vec ? 2 : 0);
-  // Cluster size: 8 bands per cluster for the float pairs when there are enough
-  // bands to fill the machine (shorter look-back chains pay off there); 4 for
-  // 8u->32s and for short/wide images (measured, DESIGN.md Sec. 6).
-  const int64_t nbands = kp.total_bands;
-  const bool byte_in = kBase<P> == P8U32S || kBase<P> == P8U32F;
-  int CL = (!byte_in && nbands >= 224) ? 8 : 4;
-  if (pl->cluster > 0) CL = pl->cluster;
-  const int cl_env = getenv_int("SAT_CLUSTER", 0);
-  if (cl_env == 1 || cl_env == 4 || cl_env == 8) CL = cl_env;
-  if (ex && CL == 1) CL = 4;  // exclusive kernels are instantiated for clusters of 4 and 8
-  if (P >= kShort) CL = 4;    // short-band kernels: clusters of 4 only
   const int ci = cluster_index(CL);
-  kp.total_tickets = (kp.total_bands + CL - 1) / CL;
   // Persistent grid: every co-resident cluster slot, but no more clusters than tickets.
   int64_t clusters =
       std::max(P >= kShort ? pl->active_short[kBase<P>] : pl->active_clusters[kBase<P>][ci][mode], 1);
-  const int cap = getenv_int("SAT_MAX_CLUSTERS", 0);
-  if (cap > 0) clusters = std::min<int64_t>(clusters, cap);
-  const int force = getenv_int("SAT_FORCE_CLUSTERS", 0);
-  if (force > 0) clusters = force;
+  if (pl->max_clusters > 0) clusters = std::min<int64_t>(clusters, pl->max_clusters);
+  if (pl->force_clusters > 0) clusters = pl->force_clusters;
   clusters = std::min<int64_t>(clusters, kp.total_tickets);
   const int64_t grid = clusters * CL;
 
@@ -200,18 +203,29 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
     e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, 4, true, true, false>, map, kp);
   } else if (ex) {
     if (CL == 4) SAT_LAUNCH_CL(4, true) else SAT_LAUNCH_CL(8, true)
-  } else if (CL == 1) SAT_LAUNCH_CL(1, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
+  } else if (CL == 2) SAT_LAUNCH_CL(2, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
 #undef SAT_LAUNCH_CL
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
 #ifdef SAT_TIMELINE
   {
-    static unsigned long long tl[1024][2 + kTlChunks];
+    static unsigned long long tl[1024][2 + kTlChunks], ta[1024][kTlChunks], tv[1024][kTlChunks],
+        t1[1024][kTlChunks], t2[1024][kTlChunks], t3[1024][kTlChunks];
     cudaStreamSynchronize(stream);
     cudaMemcpyFromSymbol(tl, g_sat_tl, sizeof(tl));
+    cudaMemcpyFromSymbol(ta, g_sat_tl_agg, sizeof(ta));
+    cudaMemcpyFromSymbol(tv, g_sat_tl_v, sizeof(tv));
+    cudaMemcpyFromSymbol(t1, g_sat_tl_ls, sizeof(t1));
+    cudaMemcpyFromSymbol(t2, g_sat_tl_lt, sizeof(t2));
+    cudaMemcpyFromSymbol(t3, g_sat_tl_ld, sizeof(t3));
     static unsigned long long zero[1024][2 + kTlChunks];
     cudaMemcpyToSymbol(g_sat_tl, zero, sizeof(zero));
+    cudaMemcpyToSymbol(g_sat_tl_agg, zero, sizeof(ta));
+    cudaMemcpyToSymbol(g_sat_tl_v, zero, sizeof(tv));
+    cudaMemcpyToSymbol(g_sat_tl_ls, zero, sizeof(ta));
+    cudaMemcpyToSymbol(g_sat_tl_lt, zero, sizeof(ta));
+    cudaMemcpyToSymbol(g_sat_tl_ld, zero, sizeof(ta));
     const char* path = getenv("SAT_TIMELINE_OUT");
     FILE* f = path ? fopen(path, "a") : nullptr;
     if (f) {
@@ -221,6 +235,16 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
       for (int64_t b = 0; b < grid && b < 1024; ++b) {
         fprintf(f, "cta %lld %llu %llu", (long long)b, tl[b][0], tl[b][1]);
         for (int c = 0; c < nc; ++c) fprintf(f, " %llu", tl[b][2 + c]);
+        fprintf(f, "\nagg %lld", (long long)b);
+        for (int c = 0; c < nc; ++c) fprintf(f, " %llu", ta[b][c]);
+        fprintf(f, "\nvup %lld", (long long)b);
+        for (int c = 0; c < nc; ++c) fprintf(f, " %llu", tv[b][c]);
+        fprintf(f, "\nls %lld", (long long)b);
+        for (int c = 0; c < nc; ++c) fprintf(f, " %llu", t1[b][c]);
+        fprintf(f, "\nlt %lld", (long long)b);
+        for (int c = 0; c < nc; ++c) fprintf(f, " %llu", t2[b][c]);
+        fprintf(f, "\nld %lld", (long long)b);
+        for (int c = 0; c < nc; ++c) fprintf(f, " %llu", t3[b][c]);
         fprintf(f, "\n");
       }
       fclose(f);
@@ -253,7 +277,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   // Every cluster draws exactly one failing ticket.
   pl->ticket_base += (uint64_t)kp.total_tickets + (uint64_t)clusters;
   pl->launches++;
-  if (getenv_int("SAT_LOG", 0))
+  if (pl->log)
     fprintf(stderr,
             "[libsat] pair=%d %lldx%lld batch=%lld tma=%d vec=%d cluster=%d grid=%lld smem=%zu "
             "epoch=%u\n",
@@ -262,9 +286,41 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   return SAT_OK;
 }
 
+static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
+                                  int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
+                                  const void* carry_in, cudaStream_t stream, const ExSpec* ex,
+                                  const ChainSpec* chain);
+
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
                   cudaStream_t stream, const ExSpec* ex, const ChainSpec* chain) {
+  // Tickets and epochs are handed out by the host per launch: a captured
+  // launch replayed from a graph would reuse them, so capture is refused.
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone)
+    return fail(SAT_ERR_UNSUPPORTED,
+                "stream capture (CUDA graphs) is not supported: libsat hands out look-back "
+                "tickets and epochs per launch on the host");
+  // Launches of one plan share its workspace: order a launch on a new stream
+  // after the plan's previous launch.
+  if (pl->has_last && pl->last_stream != stream) {
+    cudaError_t e = cudaStreamWaitEvent(stream, pl->last_ev, 0);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent(plan order)");
+  }
+  sat_status st = launch_dispatch(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+  if (st == SAT_OK) {
+    cudaError_t e = cudaEventRecord(pl->last_ev, stream);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord(plan order)");
+    pl->last_stream = stream;
+    pl->has_last = true;
+  }
+  return st;
+}
+
+static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
+                                  int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
+                                  const void* carry_in, cudaStream_t stream, const ExSpec* ex,
+                                  const ChainSpec* chain) {
   // Short, wide images: 32-row bands give only H/4 compute warps in total
   // (2 CTAs of 8 warps per SM leave most SMs idle below ~140 bands); 16-row
   // bands (2 rows per warp) double the warps in flight.
@@ -272,9 +328,8 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
   const int64_t bands32 = (h + th - 1) / th * batch;
   const bool aligned = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
                        ((uintptr_t)out % 16 == 0) && (op % 16 == 0) && (batch == 1 || ois % 16 == 0);
-  const int sh_env = getenv_int("SAT_SHORT", -1);
-  const bool use_short = !ex && aligned && getenv_int("SAT_FORCE_GENERIC", 0) == 0 &&
-                         getenv_int("SAT_CLUSTER", 0) == 0 && pl->cluster == 0 &&
+  const int sh_env = pl->short_bands;
+  const bool use_short = !ex && aligned && pl->force_generic == 0 && pl->cluster == 0 &&
                          (sh_env >= 0 ? sh_env == 1 : 2 * bands32 <= (int64_t)pl->num_sms);
   if (use_short) {
     switch (pl->pair) {
@@ -305,7 +360,12 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
 
-int cluster_index(int cl) { return cl == 1 ? 0 : (cl == 4 ? 1 : 2); }
+int cluster_index(int cl) { return cl == 2 ? 0 : cl == 4 ? 1 : 2; }
+
+int default_cluster(int base_pair, int64_t bands) {
+  const bool byte_in = base_pair == P8U32S || base_pair == P8U32F;
+  return (!byte_in && bands >= 224) ? 8 : 4;
+}
 
 int getenv_int(const char* name, int dflt) {
   const char* v = getenv(name);
@@ -332,7 +392,7 @@ static sat_status configure_cl(sat_plan_st* pl) {
   cudaError_t e0 = cudaFuncSetAttribute(sat_occupancy_proxy<P, CL>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e0 != cudaSuccess) return cuda_fail(e0, "cudaFuncSetAttribute(proxy)");
-  if constexpr (CL != 1) {
+  if constexpr (CL == 4 || CL == 8) {
     void (*fx[4])(CUtensorMap, KParams) = {
         sat_tile_kernel<P, CL, false, false, true>, sat_tile_kernel<P, CL, true, false, true>,
         sat_tile_kernel<P, CL, false, true, true>, sat_tile_kernel<P, CL, true, true, true>};
@@ -394,7 +454,7 @@ static sat_status configure_short(sat_plan_st* pl) {
 
 template <int P>
 static sat_status configure_t(sat_plan_st* pl) {
-  sat_status st = configure_cl<P, 1>(pl);
+  sat_status st = configure_cl<P, 2>(pl);
   if (st == SAT_OK) st = configure_cl<P, 4>(pl);
   if (st == SAT_OK) st = configure_cl<P, 8>(pl);
   if (st == SAT_OK) st = configure_short<P>(pl);
@@ -481,7 +541,7 @@ using namespace sat;
 
 extern "C" {
 
-int sat_version(void) { return 100; }
+int sat_version(void) { return 20000; }
 
 const char* sat_status_string(sat_status s) {
   switch (s) {
@@ -497,6 +557,8 @@ const char* sat_status_string(sat_status s) {
       return "SAT_ERR_NCCL";
     case SAT_ERR_OUT_OF_MEMORY:
       return "SAT_ERR_OUT_OF_MEMORY";
+    case SAT_ERR_TIMEOUT:
+      return "SAT_ERR_TIMEOUT";
   }
   return "SAT_ERR_UNKNOWN";
 }
@@ -534,13 +596,41 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   pl->max_w = max_w;
   pl->max_batch = max_batch;
   pl->num_sms = prop.multiProcessorCount;
+  // Environment knobs: read once, here (never on the launch path).
+  pl->force_generic = getenv_int("SAT_FORCE_GENERIC", 0);
+  {
+    const int c = getenv_int("SAT_CLUSTER", 0);
+    pl->cluster = (c == 2 || c == 4 || c == 8) ? c : 0;
+  }
+  pl->short_bands = getenv_int("SAT_SHORT", -1);
+  pl->max_clusters = getenv_int("SAT_MAX_CLUSTERS", 0);
+  pl->force_clusters = getenv_int("SAT_FORCE_CLUSTERS", 0);
+  pl->log = getenv_int("SAT_LOG", 0);
   const int64_t TH = tile_h(pair), TW = tile_w(pair);
-  pl->max_tiles = max_batch * ((max_h + TH - 1) / TH) * ((max_w + TW - 1) / TW);
-  // one status-tagged carry vector of TW elements per (ticket, chunk), 8 bytes per
-  // 32 value bits; tickets <= bands, so sizing by bands covers every cluster size
-  const size_t payload_bytes = (size_t)pl->max_tiles * TW * (out_size(pair) / 4) * 8;
+  const int64_t bands = max_batch * ((max_h + TH - 1) / TH);
+  pl->max_chunks = (max_w + TW - 1) / TW;
+  pl->max_tiles = bands * pl->max_chunks;
+  // Look-back capacity: one tagged vector (TW elements, 8 bytes per 32 value
+  // bits) per (cluster ticket, chunk).  Tickets per launch follow the cluster policy
+  // (default_cluster, or the forced size); short-band launches (<= #SMs / 2
+  // normal bands) have at most num_sms / 4 tickets.
+  int64_t tickets;
+  if (pl->cluster > 0) {
+    tickets = (bands + pl->cluster - 1) / pl->cluster;
+  } else {
+    const int base = (int)pair;
+    tickets = (std::min<int64_t>(bands, 223) + 3) / 4;
+    tickets = std::max<int64_t>(tickets, (bands + default_cluster(base, bands) - 1) / default_cluster(base, bands));
+    tickets = std::max<int64_t>(tickets, std::min<int64_t>((2 * bands + 3) / 4, (pl->num_sms + 3) / 4));
+  }
+  pl->tickets_cap = tickets;
+  const size_t payload_bytes = (size_t)tickets * pl->max_chunks * TW * (out_size(pair) / 4) * 8;
   pl->ws_bytes = 256 + payload_bytes;
   sat_status st = configure(pl);
+  if (st == SAT_OK) {
+    e = cudaEventCreateWithFlags(&pl->last_ev, cudaEventDisableTiming);
+    if (e != cudaSuccess) st = cuda_fail(e, "cudaEventCreate");
+  }
   if (st == SAT_OK) {
     e = cudaMalloc(&pl->ws, pl->ws_bytes);
     if (e != cudaSuccess) st = cuda_fail(e, "cudaMalloc(workspace)");
@@ -551,14 +641,39 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   }
   if (st != SAT_OK) {
     if (pl->ws) cudaFree(pl->ws);
+    if (pl->last_ev) cudaEventDestroy(pl->last_ev);
     delete pl;
     cudaSetDevice(prev);
     return st;
   }
   pl->counter = reinterpret_cast<unsigned long long*>(pl->ws);
+  pl->err = reinterpret_cast<uint32_t*>(static_cast<char*>(pl->ws) + 64);
   pl->payload = static_cast<char*>(pl->ws) + 256;
   cudaSetDevice(prev);
   *plan = pl;
+  return SAT_OK;
+}
+
+sat_status sat_plan_set_timeout(sat_plan plan, uint64_t ns) {
+  if (!plan || ns == 0) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL plan or zero timeout");
+  plan->spin_ns = ns;
+  return SAT_OK;
+}
+
+sat_status sat_plan_status(sat_plan plan, void* stream) {
+  if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  DeviceGuard g(plan->device);
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  uint32_t h = 0;
+  cudaError_t e = cudaMemcpyAsync(&h, plan->err, 4, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e == cudaSuccess && h != 0) e = cudaMemsetAsync(plan->err, 0, 4, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(e, "sat_plan_status");
+  if (h & 1u)
+    return fail(SAT_ERR_TIMEOUT,
+                "a carry wait exceeded the plan's timeout (a band / rank above never published); "
+                "the affected output is wrong");
   return SAT_OK;
 }
 
@@ -575,6 +690,7 @@ sat_status sat_plan_destroy(sat_plan plan) {
   cudaSetDevice(plan->device);
   host_path_release(plan);
   if (plan->ws) cudaFree(plan->ws);
+  if (plan->last_ev) cudaEventDestroy(plan->last_ev);
   cudaSetDevice(prev);
   delete plan;
   return SAT_OK;

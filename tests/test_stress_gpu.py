@@ -1,6 +1,7 @@
-"""Look-back stress: the -DSAT_DEBUG_DELAY build sleeps a pseudo-random 0..4 us
-before every carry publication, look-back round and DSMEM hand-off, so late
-predecessors, mixed aggregate/inclusive windows and retries all occur.  Run
+"""Carry-tree stress: the -DSAT_DEBUG_DELAY build sleeps a pseudo-random 0..4 us
+before every node publication, tree round and DSMEM hand-off, so late
+predecessors, half-written nodes and retries all occur (tall images reach
+tree level 3; 40 two-band frames put several whole images in one cluster).  Run
 in a subprocess (the library is chosen at import through SAT_LIBRARY)."""
 import os
 import subprocess
@@ -21,7 +22,9 @@ import paper_conf_cluster_chenwttm18_b200 as sat
 assert sat.LIB_PATH.endswith("libsat_delay.so"), sat.LIB_PATH
 bad = 0
 for (dt, H, W, N) in [(torch.uint8, 4099, 2311, 1), (torch.float32, 2500, 3000, 1),
-                      (torch.float64, 1800, 1700, 1), (torch.uint8, 1080, 900, 5)]:
+                      (torch.float64, 1800, 1700, 1), (torch.uint8, 1080, 900, 5),
+                      (torch.uint8, 9001, 700, 1), (torch.float32, 8200, 500, 1),
+                      (torch.uint8, 45, 300, 40)]:
     shape = (N, H, W) if N > 1 else (H, W)
     x = torch.empty(shape, dtype=dt, device="cuda")
     satgen.fill_device(x, seed=H + W)
@@ -42,7 +45,7 @@ print("BAD", bad)
 '''
 
 
-@pytest.mark.parametrize("cluster", ["1", "4", "8"])
+@pytest.mark.parametrize("cluster", ["2", "4", "8"])
 def test_lookback_under_injected_delays(cluster):
     if not os.path.exists(DELAY_LIB):
         pytest.skip("libsat_delay.so not built")
