@@ -189,6 +189,11 @@ sat_status sat_box_filter(sat_plan plan, const void* sat, void* out, int64_t h, 
  * loaded is reused).  Errors from NCCL map to SAT_ERR_NCCL.
  */
 
+/* Rows [*r0, *r1) of rank `rank` when h rows are split over nranks bands in
+ * rank order: the first h mod nranks ranks get one extra row (reading R14).
+ * Host-only arithmetic (no device needed).  Errors: INVALID_ARGUMENT. */
+sat_status sat_band_partition(int64_t h, int nranks, int rank, int64_t* r0, int64_t* r1);
+
 /* Bytes of an NCCL unique id (NCCL_UNIQUE_ID_BYTES). */
 #define SAT_COMM_ID_BYTES 128
 
@@ -215,35 +220,64 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
                             int64_t out_pitch_bytes, sat_pair pair, void* stream);
 
 /* ---------------------------------------------------------------------------
- * Chained row bands: the single-pass multi-GPU path.
- * Instead of a column-sum pre-pass and an all-gather, each band's kernel
+ * Chained row bands: the single-pass multi-GPU path (
+ * the paper motivates horizontal scaling but stays on one node).
+ * Instead of a column-sum pre-pass and an all-gather, the kernel of band r
  * publishes its bottom row S(r1-1, .) chunk by chunk (epoch-tagged 64-bit
- * words, the look-back payload format) straight into the receive buffer of
- * the band below -- on another GPU through peer memory -- whose top clusters
- * wait for each chunk's vector as their look-back predecessor.  Bands are read
- * once and written once (sizeof(T_A) + sizeof(T_B) bytes per pixel), and the
- * bands overlap chunk by chunk. */
+ * words, the look-back payload format) straight into the LINK of band r+1 --
+ * on another GPU through peer memory -- whose top clusters wait for each
+ * chunk's vector as the carry-in of their first band (Eq. 1 split at row r0:
+ * S(y, x) = S(r0-1, x) + SAT of rows [r0, y]).  Bands are read once and
+ * written once (sizeof(T_A) + sizeof(T_B) bytes per pixel) and overlap chunk
+ * by chunk.
+ *
+ * A link (owned by band r, sat_chain_bytes(pair, w) bytes, zero before first
+ * use, 256-byte aligned) holds ack words [nchunks] -- written by band r+1 --
+ * and two receive slots -- written by band r-1.  A call with epoch e uses
+ * slot e & 1; the band above writes a chunk of slot e & 1 only after band r
+ * has acknowledged epoch e - 2 of that chunk, so successive calls need no
+ * host or NCCL barrier: flow control is on the device.  Epochs: one value per
+ * chained SAT, the same on every band, 1, 2, 3, ... (< 2^30); restarting at 1
+ * needs zeroed links.  Waits are bounded by the plan timeout (SAT_ERR_TIMEOUT
+ * via sat_plan_status). */
 
-/* Bytes of one chain buffer (the tagged carry vectors of one row of width w). */
+/* Bytes of one chain link for rows of width w (0 for a bad pair / w <= 0). */
 size_t sat_chain_bytes(sat_pair pair, int64_t w);
 
-/* One band of a chain on this device.  chain_in (NULL for the top band) is
- * read, chain_out (NULL for the bottom band) is written: device or
- * peer-mapped pointers, 16-byte aligned, sat_chain_bytes(pair, w) bytes,
- * zero-filled once before first use.  chain_epoch in [1, 2^30) must differ
- * from the previous use of the same buffer.  The band ABOVE must be able to
- * run concurrently or earlier (e.g. same stream, earlier): a band waits in
- * its kernel for chain_in.  h, w >= 1. */
+/* Allocate (cudaMalloc, so it can be exported over CUDA IPC) and zero one link
+ * on `device`; sat_chain_link_destroy frees it. */
+sat_status sat_chain_link_create(int device, sat_pair pair, int64_t w, void** link);
+sat_status sat_chain_link_destroy(void* link);
+
+/* Bytes of a CUDA IPC memory handle (CUDA_IPC_HANDLE_SIZE). */
+#define SAT_IPC_HANDLE_BYTES 64
+
+/* Export a link created by sat_chain_link_create to another process
+ * (SAT_IPC_HANDLE_BYTES at handle_out; ship them over any transport, e.g. a
+ * torch process group), and map a peer's link into this process on `device`
+ * (peer access: NVLink between GPUs, or the same GPU).  Close with
+ * sat_chain_close_peer. */
+sat_status sat_chain_ipc_handle(const void* link, void* handle_out);
+sat_status sat_chain_open_peer(int device, const void* handle, void** peer_link);
+sat_status sat_chain_close_peer(void* peer_link);
+
+/* One band of a chain.  link_self: this band's link (required when it has a
+ * neighbour); link_above: the link of the band above (NULL for the top band)
+ * -- the carry-in comes from link_self's slot, the acknowledgement goes to
+ * link_above; link_below: the link of the band below (NULL for the bottom
+ * band) -- the bottom row goes into its slot, after link_self's ack words
+ * allow it.  Device or peer-mapped pointers.  The band above must run
+ * earlier or concurrently (a band waits in its kernel for its carry-in).
+ * h, w >= 1. */
 sat_status sat_compute_band_chained(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
                                     int64_t in_pitch_bytes, int64_t out_pitch_bytes,
-                                    const void* chain_in, void* chain_out, uint32_t chain_epoch,
-                                    sat_pair pair, void* stream);
+                                    void* link_self, void* link_above, void* link_below,
+                                    uint32_t epoch, sat_pair pair, void* stream);
 
-/* Collective: rank r holds rows [sum_{r'<r} band_h_r', +band_h) (every band
- * >= 1 row).  Receive buffers are exchanged once per width (CUDA IPC handles
- * all-gathered over NCCL; needs peer access, i.e. NVLink between the GPUs);
- * each call then does a one-int NCCL all-gather as a stream barrier (so no
- * rank overwrites a buffer its peer still reads) and ONE kernel per rank. */
+/* Collective convenience over a sat_comm: rank r holds rows
+ * [sum_{r'<r} band_h_r', +band_h) (every band >= 1 row).  Links are created
+ * and their IPC handles all-gathered over NCCL once per width; every call is
+ * then ONE kernel per rank (epochs counted by the comm, no collective). */
 sat_status sat_compute_dist_chained(sat_plan plan, sat_comm comm, const void* in_band,
                                     void* out_band, int64_t band_h, int64_t w,
                                     int64_t in_pitch_bytes, int64_t out_pitch_bytes, sat_pair pair,

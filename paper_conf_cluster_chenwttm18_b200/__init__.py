@@ -24,7 +24,8 @@ import os
 import threading
 
 __all__ = ["SatError", "Plan", "sat", "sat_host", "sat_exclusive", "sat_band", "SatComm", "sat_dist",
-           "sat_dist_chained", "sat_band_chained", "new_chain_buffer", "chain_bytes", "rect_sums",
+           "sat_dist_chained", "sat_band_chained", "new_chain_buffer", "chain_bytes", "ChainLink",
+           "PeerLink", "SatChain", "rect_sums",
            "box_filter", "band_partition",
            "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "PAIR_8U_32F", "PAIR_32S_32S", "lib",
            "LIB_PATH"]
@@ -72,7 +73,12 @@ def lib():
                     "sat_compute_exclusive": ([vp, vp, vp, i64, i64, i64, i64, i32, vp, i32, vp], i32),
                     "sat_rect_sums": ([vp, vp, i64, i64, i64, vp, i64, vp, i32, vp], i32),
                     "sat_chain_bytes": ([i32, i64], sz),
-                    "sat_compute_band_chained": ([vp, vp, vp, i64, i64, i64, i64, vp, vp, ctypes.c_uint32, i32, vp], i32),
+                    "sat_compute_band_chained": ([vp, vp, vp, i64, i64, i64, i64, vp, vp, vp, ctypes.c_uint32, i32, vp], i32),
+                    "sat_chain_link_create": ([i32, i32, i64, ctypes.POINTER(vp)], i32),
+                    "sat_chain_link_destroy": ([vp], i32),
+                    "sat_chain_ipc_handle": ([vp, vp], i32),
+                    "sat_chain_open_peer": ([i32, vp, ctypes.POINTER(vp)], i32),
+                    "sat_chain_close_peer": ([vp], i32),
                     "sat_compute_dist_chained": ([vp, vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_box_filter": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i32, vp], i32),
                     "sat_comm_unique_id": ([vp], i32),
@@ -82,6 +88,7 @@ def lib():
                     "sat_dist_acc_bytes": ([i32], sz),
                     "sat_dist_colsum": ([vp, vp, i64, i64, i64, vp, vp], i32),
                     "sat_dist_carry": ([vp, vp, i32, i32, i64, vp, vp], i32),
+                    "sat_band_partition": ([i64, i32, i32, ctypes.POINTER(i64), ctypes.POINTER(i64)], i32),
                     "sat_status_string": ([i32], ctypes.c_char_p),
                     "sat_last_error": ([], ctypes.c_char_p),
                 }
@@ -381,10 +388,12 @@ def sat_host(x, out=None, plan: Plan | None = None, device=None, stream=None):
 # Multi-GPU
 
 def band_partition(H: int, nranks: int, rank: int):
-    """Rows [r0, r1) of rank `rank` (reading R17: the first H mod P ranks get one extra row)."""
-    base, extra = divmod(H, nranks)
-    r0 = rank * base + min(rank, extra)
-    return r0, r0 + base + (1 if rank < extra else 0)
+    """Rows [r0, r1) of rank `rank` (libsat's sat_band_partition, reading R14:
+    the first H mod P ranks get one extra row)."""
+    r0, r1 = ctypes.c_int64(), ctypes.c_int64()
+    _check(lib().sat_band_partition(H, nranks, rank, ctypes.byref(r0), ctypes.byref(r1)),
+           "sat_band_partition")
+    return r0.value, r1.value
 
 
 class SatComm:
@@ -468,21 +477,87 @@ def dist_carry(gathered, rank: int, pair: int, plan: Plan | None = None, stream=
 # ---------------------------------------------------------------------------
 # Chained row bands (single-pass multi-GPU path)
 
+IPC_HANDLE_BYTES = 64
+
+
 def chain_bytes(pair: int, w: int) -> int:
-    """Bytes of one chain buffer (tagged carry vectors of a w-wide row)."""
+    """Bytes of one chain link (ack words + two receive slots) for width w."""
     return int(lib().sat_chain_bytes(pair, w))
 
 
 def new_chain_buffer(pair: int, w: int, device=None):
-    """A zero-filled, 16-byte aligned chain buffer (uint8 CUDA tensor)."""
+    """A zero-filled chain link as a uint8 CUDA tensor (single-process chains;
+    torch allocations are 512-byte aligned)."""
     torch = _torch()
     return torch.zeros(chain_bytes(pair, w), dtype=torch.uint8, device=device or "cuda")
 
 
-def sat_band_chained(x, chain_in, chain_out, epoch: int, out=None, plan: Plan | None = None,
-                     stream=None):
-    """SAT of one band of a chain: waits (in the kernel) for the band above's
-    bottom row in chain_in, publishes its own bottom row into chain_out."""
+class ChainLink:
+    """A chain link allocated by libsat (cudaMalloc, zeroed): exportable over CUDA IPC."""
+
+    def __init__(self, pair: int, w: int, device=None):
+        torch = _torch()
+        dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        h = ctypes.c_void_p()
+        _check(lib().sat_chain_link_create(dev.index, pair, w, ctypes.byref(h)), "sat_chain_link_create")
+        self.ptr, self.device = h.value, dev
+
+    def ipc_handle(self) -> bytes:
+        buf = (ctypes.c_uint8 * IPC_HANDLE_BYTES)()
+        _check(lib().sat_chain_ipc_handle(self.ptr, buf), "sat_chain_ipc_handle")
+        return bytes(buf)
+
+    def close(self):
+        if getattr(self, "ptr", None):
+            lib().sat_chain_link_destroy(self.ptr)
+            self.ptr = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class PeerLink:
+    """Another process's chain link mapped into this one (CUDA IPC)."""
+
+    def __init__(self, handle: bytes, device=None):
+        torch = _torch()
+        dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        buf = (ctypes.c_uint8 * IPC_HANDLE_BYTES).from_buffer_copy(handle)
+        h = ctypes.c_void_p()
+        _check(lib().sat_chain_open_peer(dev.index, buf, ctypes.byref(h)), "sat_chain_open_peer")
+        self.ptr = h.value
+
+    def close(self):
+        if getattr(self, "ptr", None):
+            lib().sat_chain_close_peer(self.ptr)
+            self.ptr = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def _link_ptr(link):
+    if link is None:
+        return None
+    if isinstance(link, int):
+        return link
+    if hasattr(link, "data_ptr"):
+        return link.data_ptr()
+    return link.ptr
+
+
+def sat_band_chained(x, link_self, link_above, link_below, epoch: int, out=None,
+                     plan: Plan | None = None, stream=None):
+    """SAT of one band of a chain: its carry-in row arrives (in the kernel)
+    through link_self from the band above, its bottom row goes to link_below;
+    links are tensors from new_chain_buffer, ChainLink / PeerLink objects or
+    raw device pointers (None: no such neighbour)."""
     torch = _torch()
     pair = pair_of_dtype(x.dtype, out.dtype if out is not None else None)
     H, W = x.shape
@@ -491,15 +566,46 @@ def sat_band_chained(x, chain_in, chain_out, epoch: int, out=None, plan: Plan | 
     p = plan if plan is not None else _plan_for(x.device, pair, H, W, 1)
     _check(lib().sat_compute_band_chained(
         p.handle, x.data_ptr(), out.data_ptr(), H, W, _row_layout(x)[0], _row_layout(out)[0],
-        chain_in.data_ptr() if chain_in is not None else None,
-        chain_out.data_ptr() if chain_out is not None else None, epoch, pair,
+        _link_ptr(link_self), _link_ptr(link_above), _link_ptr(link_below), epoch, pair,
         _stream_ptr(stream, x.device)), "sat_compute_band_chained")
     return out
 
 
+class SatChain:
+    """Chained row bands across the ranks of a torch process group (any
+    backend): each rank owns a ChainLink; the links' CUDA IPC handles are
+    exchanged once over the group; every call is then ONE kernel per rank with
+    device-side flow control (no collective per call)."""
+
+    def __init__(self, pair: int, w: int, group=None, device=None):
+        import torch.distributed as dist
+
+        self.rank = dist.get_rank(group)
+        self.nranks = dist.get_world_size(group)
+        self.pair, self.w = pair, w
+        self.link = ChainLink(pair, w, device)
+        self.device = self.link.device
+        handles = [None] * self.nranks
+        dist.all_gather_object(handles, self.link.ipc_handle(), group=group)
+        self.above = PeerLink(handles[self.rank - 1], self.device) if self.rank > 0 else None
+        self.below = PeerLink(handles[self.rank + 1], self.device) if self.rank + 1 < self.nranks else None
+        self.epoch = 0
+
+    def sat(self, band, out=None, plan: Plan | None = None, stream=None):
+        """This rank's band of the chained SAT (rows in rank order)."""
+        self.epoch += 1
+        return sat_band_chained(band, self.link, self.above, self.below, self.epoch, out=out,
+                                plan=plan, stream=stream)
+
+    def close(self):
+        for l in (self.above, self.below, self.link):
+            if l is not None:
+                l.close()
+
+
 def sat_dist_chained(band, comm: SatComm, out=None, plan: Plan | None = None, stream=None):
     """Row-banded SAT across ranks with chained carries over peer memory (one
-    kernel per rank, no column-sum pass)."""
+    kernel per rank, no column-sum pass); links bootstrapped over the NCCL comm."""
     torch = _torch()
     pair = pair_of_dtype(band.dtype, out.dtype if out is not None else None)
     if out is None:

@@ -20,6 +20,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <vector>
 #include <mutex>
 
 #include "nccl.h"
@@ -341,16 +342,17 @@ sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, 
 
 using namespace sat;
 
-// Chained-band state (sat_compute_dist_chained): this rank's receive buffer
-// for the carry vectors of the rank above, and the peer-mapped receive buffer
-// of the rank below (CUDA IPC over NVLink), exchanged once per width.
+// Chained-band state (sat_compute_dist_chained): this rank's link and the
+// peer-mapped links of the ranks above and below (CUDA IPC over NVLink),
+// exchanged once per width; calls then need no collective at all (the links'
+// ack words give device-side flow control, see KParams).
 struct ChainBufs {
   int64_t w = 0;
   size_t bytes = 0;
-  void* recv = nullptr;       // own, written by rank - 1
-  void* peer_recv = nullptr;  // rank + 1's, opened through its IPC handle
-  void* hdl_dev = nullptr;    // [nranks] IPC handles (allgather staging)
-  int* flag_dev = nullptr;    // [nranks] barrier words
+  void* link = nullptr;        // own link (ack words + 2 receive slots)
+  void* peer_above = nullptr;  // rank - 1's link
+  void* peer_below = nullptr;  // rank + 1's link
+  void* hdl_dev = nullptr;     // [nranks] IPC handles (allgather staging)
   uint32_t epoch = 0;
 };
 
@@ -362,10 +364,10 @@ struct sat_comm_st {
 };
 
 static void free_chain(ChainBufs& c) {
-  if (c.peer_recv) cudaIpcCloseMemHandle(c.peer_recv);
-  if (c.recv) cudaFree(c.recv);
+  if (c.peer_above) cudaIpcCloseMemHandle(c.peer_above);
+  if (c.peer_below) cudaIpcCloseMemHandle(c.peer_below);
+  if (c.link) cudaFree(c.link);
   if (c.hdl_dev) cudaFree(c.hdl_dev);
-  if (c.flag_dev) cudaFree(c.flag_dev);
   c = ChainBufs();
 }
 
@@ -395,6 +397,16 @@ static sat_status ensure_bufs(DistBufs& b, int64_t w, int nranks) {
 }
 
 extern "C" {
+
+sat_status sat_band_partition(int64_t h, int nranks, int rank, int64_t* r0, int64_t* r1) {
+  if (!r0 || !r1 || h < 0 || nranks < 1 || rank < 0 || rank >= nranks)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "bad partition request (h=%lld, rank %d of %d)",
+                (long long)h, rank, nranks);
+  const int64_t base = h / nranks, extra = h % nranks;
+  *r0 = rank * base + std::min<int64_t>(rank, extra);
+  *r1 = *r0 + base + (rank < extra ? 1 : 0);
+  return SAT_OK;
+}
 
 sat_status sat_comm_unique_id(void* id_out) {
   if (!id_out) return fail(SAT_ERR_INVALID_ARGUMENT, "id_out is NULL");
@@ -511,30 +523,99 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
 }
 
 
-size_t sat_chain_bytes(sat_pair pair, int64_t w) {
-  if (w <= 0 || (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F &&
-                 pair != SAT_8U_32F && pair != SAT_32S_32S))
-    return 0;
-  // one tagged 64-bit word per 32-bit half of each output element, per chunk
+static bool valid_pair(sat_pair pair) {
+  return pair == SAT_8U_32S || pair == SAT_32F_32F || pair == SAT_64F_64F || pair == SAT_8U_32F ||
+         pair == SAT_32S_32S;
+}
+
+// Link layout: [ack words: nchunks u32, padded to 256 B][slot 0][slot 1], a
+// slot = one tagged 64-bit word per 32-bit half of each output element, per chunk.
+static size_t chain_ack_bytes(sat_pair pair, int64_t w) {
+  const int64_t nch = (w + tile_w(pair) - 1) / tile_w(pair);
+  return (size_t)((nch * 4 + 255) / 256 * 256);
+}
+static size_t chain_slot_bytes(sat_pair pair, int64_t w) {
   const int64_t tw = tile_w(pair);
   return (size_t)((w + tw - 1) / tw) * (size_t)tw * out_size(pair) * 2;
 }
 
+size_t sat_chain_bytes(sat_pair pair, int64_t w) {
+  if (w <= 0 || !valid_pair(pair)) return 0;
+  return chain_ack_bytes(pair, w) + 2 * chain_slot_bytes(pair, w);
+}
+
+sat_status sat_chain_link_create(int device, sat_pair pair, int64_t w, void** link) {
+  if (!link) return fail(SAT_ERR_INVALID_ARGUMENT, "link out-pointer is NULL");
+  *link = nullptr;
+  if (w <= 0 || !valid_pair(pair)) return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair or width");
+  DeviceGuard g(device);
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, sat_chain_bytes(pair, w));
+  if (e == cudaSuccess) e = cudaMemset(p, 0, sat_chain_bytes(pair, w));
+  if (e != cudaSuccess) {
+    if (p) cudaFree(p);
+    return cuda_fail(e, "sat_chain_link_create");
+  }
+  *link = p;
+  return SAT_OK;
+}
+
+sat_status sat_chain_link_destroy(void* link) {
+  if (!link) return SAT_OK;
+  cudaError_t e = cudaFree(link);
+  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "sat_chain_link_destroy");
+}
+
+sat_status sat_chain_ipc_handle(const void* link, void* handle_out) {
+  if (!link || !handle_out) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
+  static_assert(sizeof(cudaIpcMemHandle_t) == SAT_IPC_HANDLE_BYTES, "IPC handle size");
+  cudaIpcMemHandle_t h;
+  cudaError_t e = cudaIpcGetMemHandle(&h, const_cast<void*>(link));
+  if (e != cudaSuccess) return cuda_fail(e, "cudaIpcGetMemHandle");
+  memcpy(handle_out, &h, sizeof(h));
+  return SAT_OK;
+}
+
+sat_status sat_chain_open_peer(int device, const void* handle, void** peer_link) {
+  if (!handle || !peer_link) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
+  *peer_link = nullptr;
+  DeviceGuard g(device);
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, sizeof(h));
+  cudaError_t e = cudaIpcOpenMemHandle(peer_link, h, cudaIpcMemLazyEnablePeerAccess);
+  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "cudaIpcOpenMemHandle");
+}
+
+sat_status sat_chain_close_peer(void* peer_link) {
+  if (!peer_link) return SAT_OK;
+  cudaError_t e = cudaIpcCloseMemHandle(peer_link);
+  return e == cudaSuccess ? SAT_OK : cuda_fail(e, "cudaIpcCloseMemHandle");
+}
+
 sat_status sat_compute_band_chained(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
                                     int64_t in_pitch_bytes, int64_t out_pitch_bytes,
-                                    const void* chain_in, void* chain_out, uint32_t chain_epoch,
-                                    sat_pair pair, void* stream) {
+                                    void* link_self, void* link_above, void* link_below,
+                                    uint32_t epoch, sat_pair pair, void* stream) {
   if (h <= 0 || w <= 0) return fail(SAT_ERR_INVALID_ARGUMENT, "a chained band needs h, w >= 1");
-  if (chain_epoch == 0 || chain_epoch >= (1u << 30))
-    return fail(SAT_ERR_INVALID_ARGUMENT, "chain_epoch must be in [1, 2^30)");
-  if (((uintptr_t)chain_in | (uintptr_t)chain_out) % 16 != 0)
-    return fail(SAT_ERR_INVALID_ARGUMENT, "chain buffers must be 16-byte aligned");
+  if (epoch == 0 || epoch >= (1u << 30))
+    return fail(SAT_ERR_INVALID_ARGUMENT, "epoch must be in [1, 2^30)");
+  if ((link_above || link_below) && !link_self)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "a band with a neighbour needs its own link");
+  if (((uintptr_t)link_self | (uintptr_t)link_above | (uintptr_t)link_below) % 256 != 0)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "chain links must be 256-byte aligned");
   bool empty = false;
   sat_status st = validate(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
                            h * in_pitch_bytes, h * out_pitch_bytes, 1, pair, &empty);
   if (st != SAT_OK || empty) return st;
   DeviceGuard g(plan->device);
-  const ChainSpec chain{chain_in, chain_out, chain_epoch};
+  const size_t ab = chain_ack_bytes(pair, w), sb = chain_slot_bytes(pair, w);
+  const size_t slot = ab + (size_t)(epoch & 1u) * sb;
+  ChainSpec chain;
+  chain.in = link_above ? static_cast<const char*>(link_self) + slot : nullptr;
+  chain.ack_out = link_above ? static_cast<uint32_t*>(link_above) : nullptr;
+  chain.out = link_below ? static_cast<char*>(link_below) + slot : nullptr;
+  chain.ack_in = link_below ? static_cast<const uint32_t*>(link_self) : nullptr;
+  chain.epoch = epoch;
   return launch(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes, h * in_pitch_bytes,
                 h * out_pitch_bytes, 1, nullptr, static_cast<cudaStream_t>(stream), nullptr, &chain);
 }
@@ -558,52 +639,51 @@ sat_status sat_compute_dist_chained(sat_plan plan, sat_comm comm, const void* in
                   band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1, nullptr, s);
   ChainBufs& c = comm->chain;
   const size_t bytes = sat_chain_bytes(pair, w);
-  if (c.bytes < bytes) {  // (re)build: collective, every rank calls with the same w
+  if (c.bytes != bytes || c.w != w) {  // (re)build: collective, every rank calls with the same w
     cudaStreamSynchronize(s);
     free_chain(c);
-    cudaError_t e = cudaMalloc(&c.recv, bytes);
-    if (e == cudaSuccess) e = cudaMemset(c.recv, 0, bytes);
-    if (e == cudaSuccess) e = cudaMalloc(&c.hdl_dev, (size_t)comm->nranks * sizeof(cudaIpcMemHandle_t));
-    if (e == cudaSuccess) e = cudaMalloc(&c.flag_dev, (size_t)comm->nranks * 2 * sizeof(int));
-    cudaIpcMemHandle_t mine;
-    if (e == cudaSuccess) e = cudaIpcGetMemHandle(&mine, c.recv);
-    if (e == cudaSuccess)
-      e = cudaMemcpy(static_cast<char*>(c.hdl_dev) + comm->rank * sizeof(mine), &mine, sizeof(mine),
-                     cudaMemcpyHostToDevice);
+    const size_t hb = sizeof(cudaIpcMemHandle_t);
+    st = sat_chain_link_create(comm->device, pair, w, &c.link);
+    if (st != SAT_OK) return st;
+    cudaError_t e = cudaMalloc(&c.hdl_dev, (size_t)comm->nranks * hb);
+    unsigned char mine[SAT_IPC_HANDLE_BYTES];
+    if (e == cudaSuccess) {
+      st = sat_chain_ipc_handle(c.link, mine);
+      if (st != SAT_OK) {
+        free_chain(c);
+        return st;
+      }
+      e = cudaMemcpyAsync(static_cast<char*>(c.hdl_dev) + comm->rank * hb, mine, hb,
+                          cudaMemcpyHostToDevice, s);
+    }
     if (e != cudaSuccess) {
       free_chain(c);
-      return cuda_fail(e, "chain buffers");
+      return cuda_fail(e, "chain handle staging");
     }
-    ncclResult_t r = nccl().AllGather(static_cast<char*>(c.hdl_dev) + comm->rank * sizeof(mine),
-                                      c.hdl_dev, sizeof(mine), ncclUint8, comm->comm, s);
+    ncclResult_t r = nccl().AllGather(static_cast<char*>(c.hdl_dev) + comm->rank * hb, c.hdl_dev, hb,
+                                      ncclUint8, comm->comm, s);
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather(ipc handles)");
-    e = cudaStreamSynchronize(s);
-    if (e == cudaSuccess && comm->rank + 1 < comm->nranks) {
-      cudaIpcMemHandle_t below;
-      e = cudaMemcpy(&below, static_cast<char*>(c.hdl_dev) + (comm->rank + 1) * sizeof(below),
-                     sizeof(below), cudaMemcpyDeviceToHost);
-      if (e == cudaSuccess) e = cudaIpcOpenMemHandle(&c.peer_recv, below, cudaIpcMemLazyEnablePeerAccess);
-    }
+    std::vector<unsigned char> all((size_t)comm->nranks * hb);
+    e = cudaMemcpyAsync(all.data(), c.hdl_dev, all.size(), cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e != cudaSuccess) {
       free_chain(c);
-      return cuda_fail(e, "chain peer mapping");
+      return cuda_fail(e, "chain handle exchange");
+    }
+    if (comm->rank > 0) st = sat_chain_open_peer(comm->device, &all[(comm->rank - 1) * hb], &c.peer_above);
+    if (st == SAT_OK && comm->rank + 1 < comm->nranks)
+      st = sat_chain_open_peer(comm->device, &all[(comm->rank + 1) * hb], &c.peer_below);
+    if (st != SAT_OK) {
+      free_chain(c);
+      return st;
     }
     c.bytes = bytes;
     c.w = w;
+    c.epoch = 0;
   }
-  if (++c.epoch >= (1u << 30)) {  // tags hold 30 epoch bits: clear and restart (collective)
-    cudaError_t e = cudaMemsetAsync(c.recv, 0, c.bytes, s);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(chain)");
-    c.epoch = 1;
-  }
-  // Barrier on the stream: no rank overwrites its peer's receive buffer for this
-  // call before that peer has finished reading it in the previous call.
-  ncclResult_t r = nccl().AllGather(c.flag_dev + comm->rank, c.flag_dev + comm->nranks, 1,
-                                    ncclInt32, comm->comm, s);
-  if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather(barrier)");
-  const ChainSpec chain{comm->rank > 0 ? c.recv : nullptr, c.peer_recv, c.epoch};
-  return launch(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
-                band_h * in_pitch_bytes, band_h * out_pitch_bytes, 1, nullptr, s, nullptr, &chain);
+  if (++c.epoch >= (1u << 30)) return fail(SAT_ERR_UNSUPPORTED, "chain epochs exhausted: recreate the comm");
+  return sat_compute_band_chained(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,
+                                  c.link, c.peer_above, c.peer_below, c.epoch, pair, stream);
 }
 
 }  // extern "C"

@@ -71,8 +71,10 @@ struct ExSpec {
 // Chained bands: per-chunk tagged carry vectors in (from the band above) and
 // out (this band's bottom row, for the band below); see KParams.
 struct ChainSpec {
-  const void* in;
-  void* out;
+  const void* in;        // this call's receive slot (band above publishes), or NULL
+  void* out;             // the band below's receive slot, or NULL
+  uint32_t* ack_out;     // the band above's ack words (written after reading `in`)
+  const uint32_t* ack_in;  // this band's ack words (read before writing `out`)
   uint32_t epoch;
 };
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,

@@ -252,8 +252,14 @@ struct KParams {
   // chunk as an epoch-tagged vector (payload layout) written by the kernel of
   // the band above -- possibly on another GPU through peer memory -- and this
   // band's bottom row S(r1-1, .) is published the same way for the band below.
-  const uint64_t* chain_in;              // [nchunks][kVecWords] or NULL
-  uint64_t* chain_out;                   // [nchunks][kVecWords] or NULL
+  // Flow control (double-buffered slots): the band below acknowledges each
+  // consumed chunk by writing the epoch into the upper band's ack word; a band
+  // overwrites a slot (epoch e, slot e & 1) only after the band below has
+  // acknowledged epoch e - 2 of that chunk.  No host or NCCL barrier per call.
+  const uint64_t* chain_in;              // this call's receive slot [nchunks][kVecWords] or NULL
+  uint64_t* chain_out;                   // the band below's receive slot or NULL
+  uint32_t* chain_ack_out;               // the band above's ack words [nchunks] (with chain_in)
+  const uint32_t* chain_ack_in;          // this band's ack words (with chain_out)
   uint32_t chain_epoch;                  // >= 1; tag = (chain_epoch << 2) | kStIncl
   // Bounded waits: a cross-CTA / cross-GPU carry wait that exceeds spin_ns
   // sets bit 0 of *err, takes zeros and lets the launch finish (the host
@@ -1051,6 +1057,23 @@ __device__ __forceinline__ void chain_publish(const KParams& p, int32_t chunk,
                                               int lane) {
   using C = Cfg<P>;
   uint64_t* row = p.chain_out + (int64_t)chunk * kVecWords<P>;
+  // The slot was last used by epoch e - 2: wait until the band below consumed it.
+  if (p.chain_ack_in != nullptr && p.chain_epoch > 2) {
+    const uint32_t need = p.chain_epoch - 2;
+    const uint64_t t_start = gclock();
+    for (;;) {
+      uint32_t a = 0;
+      if (lane == 0)
+        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(a) : "l"(p.chain_ack_in + chunk) : "memory");
+      a = __shfl_sync(kFull, a, 0);
+      if ((int32_t)(a - need) >= 0) break;
+      if (gclock() - t_start > p.spin_ns) {
+        if (lane == 0) flag_timeout(p);
+        break;
+      }
+      __nanosleep(64);
+    }
+  }
 #pragma unroll
   for (int g = 0; g < C::G; ++g) {
     uint64_t w[4];
@@ -1082,6 +1105,11 @@ __device__ __forceinline__ void chain_wait(const KParams& p, int32_t chunk,
     if (__all_sync(kFull, ok)) {
 #pragma unroll
       for (int g = 0; g < C::G; ++g) Tag<kBase<P>>::dec(w[g], V[g]);
+      // every lane holds its words: release the slot to the band above
+      if (lane == 0 && p.chain_ack_out != nullptr)
+        asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p.chain_ack_out + chunk),
+                     "r"(p.chain_epoch)
+                     : "memory");
       return;
     }
     if (gclock() - t_start > p.spin_ns) {  // the band above never published: zeros, flag

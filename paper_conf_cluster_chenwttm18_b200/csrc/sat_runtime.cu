@@ -108,6 +108,8 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.nval_bits = ex ? ex->nval_bits : 0;
   kp.chain_in = chain ? static_cast<const uint64_t*>(chain->in) : nullptr;
   kp.chain_out = chain ? static_cast<uint64_t*>(chain->out) : nullptr;
+  kp.chain_ack_out = chain ? chain->ack_out : nullptr;
+  kp.chain_ack_in = chain ? chain->ack_in : nullptr;
   kp.chain_epoch = chain ? chain->epoch : 0;
 
   CUtensorMap map;

@@ -1,8 +1,10 @@
 """Chained row bands (sat_compute_band_chained): each
-band's kernel publishes its bottom row per chunk into the next band's chain
-buffer, whose top clusters wait for it.  On one GPU the "ranks" run in order
-on one stream (the same device code that peers run concurrently on separate
-GPUs); results against the oracle, bars as everywhere."""
+band's kernel publishes its bottom row per chunk into the next band's link,
+whose top clusters wait for it; the lower band acknowledges each chunk so the
+upper band may reuse the slot two epochs later.  On one GPU the "ranks" run in
+order on one stream, or concurrently on separate streams (the same device code
+that peers run on separate GPUs); results against the oracle, bars as
+everywhere."""
 import numpy as np
 import pytest
 
@@ -36,21 +38,29 @@ def _check(got, ref, d, what):
         assert rel <= TOL[d], f"{what}: rel err {rel}"
 
 
+def _links(sat, pair, W, P):
+    return [sat.new_chain_buffer(pair, W) for _ in range(P)]
+
+
+def _band(sat, x, out, links, r, P, ep, **kw):
+    return sat.sat_band_chained(x, links[r], links[r - 1] if r > 0 else None,
+                                links[r + 1] if r < P - 1 else None, ep, out=out, **kw)
+
+
 def _run_chain(d, H, W, P, epochs=(1,), short=None, monkeypatch=None):
     torch, sat = _t(), _sat()
     if short is not None:
         monkeypatch.setenv("SAT_SHORT", short)
-    x = torch.empty((H, W), dtype=_tdt(d), device="cuda")
-    satgen.fill_device(x, seed=77 + P)
-    pair = sat.pair_of_dtype(x.dtype)
-    bufs = [sat.new_chain_buffer(pair, W) for _ in range(P - 1)]
+    pair = sat.pair_of_dtype(_tdt(d))
+    links = _links(sat, pair, W, P)
     out = torch.empty((H, W), dtype=sat.out_dtype(pair), device="cuda")
     for ep in epochs:
+        x = torch.empty((H, W), dtype=_tdt(d), device="cuda")
+        satgen.fill_device(x, seed=77 + P + ep)  # new data every epoch: slots must not mix
         out.fill_(0)
         for r in range(P):
             r0, r1 = sat.band_partition(H, P, r)
-            sat.sat_band_chained(x[r0:r1], bufs[r - 1] if r > 0 else None,
-                                 bufs[r] if r < P - 1 else None, ep, out=out[r0:r1])
+            _band(sat, x[r0:r1], out[r0:r1], links, r, P, ep)
         torch.cuda.synchronize()
         _check(out.cpu().numpy(), oracle.sat(x.cpu().numpy()), d, f"P={P} {H}x{W} epoch {ep}")
 
@@ -62,9 +72,10 @@ def test_chained_bands(d, P):
 
 
 def test_chained_bands_epoch_reuse_and_tiny_bands():
-    """Buffers reused with increasing epochs; bands of one row and of one
-    chunk; W a multiple of the tile width."""
-    _run_chain(np.uint8, 37, 512, 5, epochs=(1, 2, 3))
+    """Links reused with increasing epochs (both slots, acknowledgements);
+    bands of one row and of one chunk; W a multiple of the tile width."""
+    _run_chain(np.uint8, 37, 512, 5, epochs=(1, 2, 3, 4, 5, 6))
+    _run_chain(np.float32, 700, 900, 3, epochs=(1, 2, 3))
     _run_chain(np.float64, 9, 64, 9)
     _run_chain(np.float32, 300, 1, 4)
 
@@ -83,11 +94,10 @@ def test_chained_full_size_8u_16384sq_sampled():
     x = torch.empty((H, W), dtype=torch.uint8, device="cuda")
     satgen.fill_device(x, seed=1001)
     out = torch.empty((H, W), dtype=torch.int32, device="cuda")
-    bufs = [sat.new_chain_buffer(0, W) for _ in range(P - 1)]
+    links = _links(sat, 0, W, P)
     for r in range(P):
         r0, r1 = sat.band_partition(H, P, r)
-        sat.sat_band_chained(x[r0:r1], bufs[r - 1] if r > 0 else None,
-                             bufs[r] if r < P - 1 else None, 1, out=out[r0:r1])
+        _band(sat, x[r0:r1], out[r0:r1], links, r, P, 1)
     torch.cuda.synchronize()
     rows = [0, 4095, 4096, 8191, 8192, 12287, 12288, H - 1]
     ref = oracle.sat_gen_rows(0, H, W, rows, seed=1001)
@@ -95,21 +105,76 @@ def test_chained_full_size_8u_16384sq_sampled():
 
 
 def test_chained_invalid_arguments():
-    import ctypes
     torch, sat = _t(), _sat()
     L = sat.lib()
     x = torch.zeros((64, 64), dtype=torch.uint8, device="cuda")
     o = torch.zeros((64, 64), dtype=torch.int32, device="cuda")
     b = sat.new_chain_buffer(0, 64)
+    c = sat.new_chain_buffer(0, 64)
     p = sat.Plan(0, 64, 64, 1)
-    assert L.sat_compute_band_chained(p.handle, x.data_ptr(), o.data_ptr(), 64, 64, 64, 256,
-                                      None, b.data_ptr(), 0, 0, None) == 1  # epoch 0
+    args = (p.handle, x.data_ptr(), o.data_ptr(), 64, 64, 64, 256)
+    assert L.sat_compute_band_chained(*args, b.data_ptr(), None, c.data_ptr(), 0, 0, None) == 1  # epoch 0
     assert L.sat_compute_band_chained(p.handle, x.data_ptr(), o.data_ptr(), 0, 64, 64, 256,
-                                      None, b.data_ptr(), 1, 0, None) == 1  # empty band
-    assert L.sat_compute_band_chained(p.handle, x.data_ptr(), o.data_ptr(), 64, 64, 64, 256,
-                                      None, b.data_ptr() + 8, 1, 0, None) == 1  # alignment
-    assert sat.chain_bytes(0, 257) == 2 * 256 * 4 * 2
+                                      b.data_ptr(), None, c.data_ptr(), 1, 0, None) == 1  # empty band
+    assert L.sat_compute_band_chained(*args, b.data_ptr(), None, c.data_ptr() + 16, 1, 0, None) == 1  # alignment
+    assert L.sat_compute_band_chained(*args, None, None, c.data_ptr(), 1, 0, None) == 1  # no own link
+    # 257 columns = 2 chunks of 256: 256 bytes of ack words + 2 slots of 2 x 256 x 8 bytes
+    assert sat.chain_bytes(0, 257) == 256 + 2 * (2 * 256 * 4 * 2)
     p.close()
+
+
+def test_chained_missing_upstream_band_times_out():
+    """A band whose band above never runs: its bounded wait runs out, the launch
+    finishes (no hung GPU) and sat_plan_status reports SAT_ERR_TIMEOUT; the plan
+    works normally afterwards."""
+    torch, sat = _t(), _sat()
+    H, W = 256, 1000
+    x = torch.ones((H, W), dtype=torch.uint8, device="cuda")
+    links = _links(sat, 0, W, 2)
+    p = sat.Plan(0, H, W, 1)
+    p.set_timeout(20_000_000)  # 20 ms
+    sat.sat_band_chained(x, links[1], links[0], None, 1, plan=p)  # band 1 of 2; band 0 never runs
+    with pytest.raises(sat.SatError) as ei:
+        p.status()
+    assert ei.value.status == 6  # SAT_ERR_TIMEOUT
+    p.status()  # cleared
+    y = sat.sat(x, plan=p)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy(), oracle.sat(x.cpu().numpy()))
+    p.close()
+
+
+def test_chained_flow_control_concurrent_epochs(monkeypatch):
+    """Two bands on two streams, three epochs each, the lower stream enqueued
+    late: the upper band's epoch-3 kernel must wait (on the device) for the
+    lower band to acknowledge epoch 1 of every chunk before reusing the slot.
+    Every epoch has its own input; every output checked."""
+    torch, sat = _t(), _sat()
+    monkeypatch.setenv("SAT_MAX_CLUSTERS", "16")  # both bands co-resident
+    monkeypatch.setenv("SAT_SHORT", "0")
+    H, W, P, E = 2 * 1024, 6000, 2, 3
+    pair = 0
+    links = _links(sat, pair, W, P)
+    xs = []
+    for e in range(E):
+        x = torch.empty((H, W), dtype=torch.uint8, device="cuda")
+        satgen.fill_device(x, seed=500 + e)
+        xs.append(x)
+    outs = [torch.zeros((H, W), dtype=torch.int32, device="cuda") for _ in range(E)]
+    plans = [sat.Plan(pair, H, W, 1) for _ in range(P)]
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    torch.cuda.synchronize()
+    for r in range(P):  # upper band's three epochs first, then the lower band's
+        r0, r1 = sat.band_partition(H, P, r)
+        for e in range(E):
+            with torch.cuda.stream(streams[r]):
+                _band(sat, xs[e][r0:r1], outs[e][r0:r1], links, r, P, e + 1, plan=plans[r],
+                      stream=streams[r])
+    torch.cuda.synchronize()
+    for pl in plans:
+        pl.status()
+    for e in range(E):
+        assert np.array_equal(outs[e].cpu().numpy(), oracle.sat(xs[e].cpu().numpy())), f"epoch {e + 1}"
 
 
 @pytest.mark.parametrize("d", [np.uint8, np.float32])
@@ -127,7 +192,7 @@ def test_chained_bands_concurrent_streams(monkeypatch, d):
     x = torch.empty((H, W), dtype=_tdt(d), device="cuda")
     satgen.fill_device(x, seed=91)
     pair = sat.pair_of_dtype(x.dtype)
-    bufs = [sat.new_chain_buffer(pair, W) for _ in range(P - 1)]
+    links = _links(sat, pair, W, P)
     out = torch.empty((H, W), dtype=sat.out_dtype(pair), device="cuda")
     plans = [sat.Plan(pair, H, W, 1) for _ in range(P)]
     streams = [torch.cuda.Stream() for _ in range(P)]
@@ -135,8 +200,6 @@ def test_chained_bands_concurrent_streams(monkeypatch, d):
     for r in reversed(range(P)):  # lowest band first: it must wait for the others
         r0, r1 = sat.band_partition(H, P, r)
         with torch.cuda.stream(streams[r]):
-            sat.sat_band_chained(x[r0:r1], bufs[r - 1] if r > 0 else None,
-                                 bufs[r] if r < P - 1 else None, 1, out=out[r0:r1],
-                                 plan=plans[r], stream=streams[r])
+            _band(sat, x[r0:r1], out[r0:r1], links, r, P, 1, plan=plans[r], stream=streams[r])
     torch.cuda.synchronize()
     _check(out.cpu().numpy(), oracle.sat(x.cpu().numpy()), d, "concurrent chain")

@@ -1,12 +1,15 @@
-"""Multi-process host logic of the row-banded path, on CPU with gloo (world 2).
+"""Multi-process host logic of the row-banded paths, on CPU with gloo (world 2).
 
-The CUDA steps of sat_compute_dist are covered on one GPU by
-test_parity_gpu.py::test_dist_virtual_ranks.  Here two real processes check
-what crosses process boundaries: the band partition (reading R14), the NCCL
-unique-id bootstrap over a torch process group (SatComm's protocol), and the
-carry algebra of SURVEY Sec. 8(e) -- each rank's column totals are
-all-gathered, the exclusive prefix over lower ranks is scanned horizontally,
-and the result must equal the oracle's row S(r0 - 1, .).
+The CUDA steps of sat_compute_dist / the chained bands are covered on one GPU
+by test_parity_gpu.py::test_dist_virtual_ranks, tests/test_chain_gpu.py and the
+two-process tests/test_chain_ipc_gpu.py.  Here two real processes check what
+crosses process boundaries, driving libsat's own host code where it has any:
+the band partition (libsat's sat_band_partition, reading R14), the NCCL
+unique-id bootstrap over a torch process group (SatComm's protocol), the
+all_gather_object exchange that SatChain uses for its IPC handles, and the carry
+algebra of SURVEY Sec. 8(e) -- each rank's column totals are all-gathered, the
+exclusive prefix over lower ranks is scanned horizontally, and the result must
+equal the oracle's row S(r0 - 1, .).
 """
 import os
 import socket
@@ -70,6 +73,10 @@ def _worker(rank, world, port, q):
             ok_id = ids[0] == ids[1] and any(ids[0])
         except RuntimeError:
             ok_id = "skip"
+        # 5. the SatChain handle exchange pattern (fixed-size byte strings, rank order)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, bytes([rank]) * sat.IPC_HANDLE_BYTES)
+        ok_id = ok_id if blobs == [bytes([r]) * sat.IPC_HANDLE_BYTES for r in range(world)] else False
         q.put((rank, spans, ok_carry, ok_id))
         dist.destroy_process_group()
     except Exception as e:  # report, don't hang the parent
@@ -94,3 +101,19 @@ def test_row_band_protocol_two_ranks():
         assert ok_carry, f"rank {rank}: carry row != oracle S(r0-1, .)"
         if ok_id != "skip":
             assert ok_id, f"rank {rank}: unique id not shared"
+
+
+def test_band_partition_host_code():
+    """libsat's partition (host-only C): contiguous, covering, sizes differ by
+    at most one with the larger bands first (R14); invalid requests refused."""
+    for h in (0, 1, 5, 257, 65536, 65537):
+        for n in (1, 2, 3, 8):
+            spans = [sat.band_partition(h, n, r) for r in range(n)]
+            assert spans[0][0] == 0 and spans[-1][1] == h
+            assert all(spans[i][1] == spans[i + 1][0] for i in range(n - 1))
+            sizes = [b - a for a, b in spans]
+            assert max(sizes) - min(sizes) <= (1 if h else 0) and sizes == sorted(sizes, reverse=True)
+    with pytest.raises(sat.SatError):
+        sat.band_partition(10, 2, 2)
+    with pytest.raises(sat.SatError):
+        sat.band_partition(-1, 2, 0)
