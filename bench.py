@@ -5,16 +5,29 @@ achieved HBM GB/s vs the HBM roofline).
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
                     [--workload NAME] [--no-sweep]
 
-Workload (N=1 headline, BASELINE.json configs[1]): the 16384 x 16384 8u->32s
-image of the size sweep, synthetic (satgen, seed 1001).  Under torchrun
-(N > 1) every rank computes its own independent 16384^2 image (image index =
-rank): the path shards by image with no data-path collective ("weak").
+Headline (N=1: BASELINE.json configs[1] at its largest size): the 16384 x
+16384 8u->32s image of the size sweep, synthetic (satgen, seed 1001).  Under
+torchrun (N > 1) every rank computes its own independent 16384^2 image (image
+index = rank): the path shards by image with no data-path collective ("weak").
 
 A step = one sat_compute over the whole image (one kernel launch).  Inputs
 (268 MB in + 1.07 GB out per step) exceed the 126 MB L2, so no flush is
-needed for the headline; the sweep entries below 4096^2 flush L2 between steps.
-Timing: CUDA events on the launching stream, barrier + synchronize around the
-K timed steps, max over ranks.  rank 0 prints ONE JSON line.
+needed for the headline; the sweep entries below 4 x L2 flush L2 between
+steps.  Timing: CUDA events on the launching stream, barrier + synchronize
+around the K timed steps, max over ranks.  The NVML clock sampler runs through
+a >= 250 ms soak of the same launches immediately before the timed steps and
+through the timed steps (so the clock record covers a sustained load, not just
+the few ms of K headline steps).
+
+The same JSON line also carries, at every N:
+  sharded_batch : BASELINE configs[2] -- 1024 1080x1920 8u frames split
+                  1024/N per rank (strong scaling), aggregate Gpx/s;
+  banded        : BASELINE configs[3] -- one 65536^2 32f image in N row bands,
+                  two legs: "colsum" (column sums -> ncclAllGather -> carry ->
+                  band SAT, each phase timed) and "chained" (one kernel per
+                  rank, bottom rows published into the next GPU's link), plus
+                  a cross-check of the two legs' outputs (different algorithms,
+                  so agreement within the 1e-4 bar is evidence for both).
 
 --impl reference times the CPU oracle (oracle/, single thread, as it stands)
 on the same workload, one full image per step (rank 0 only).
@@ -75,7 +88,7 @@ def ncu_traffic(workload):
 class ClockSampler:
     """Samples SM clock + throttle reasons via NVML during the timed region."""
 
-    def __init__(self, index: int, period_s: float = 0.002):
+    def __init__(self, index: int, period_s: float = 0.001):
         self.index, self.period = index, period_s
         self.samples, self.reasons = [], set()
         self.max_mhz = None
@@ -284,19 +297,27 @@ def run_ours(args, workload, rank, world, local_rank):
         else:
             plan.compute_ptr(x.data_ptr(), out.data_ptr(), H, W, W * IN_B[pair], W * OUT_B[pair], s)
 
+    wa, wb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    wa.record(s)
     for _ in range(args.warmup):
         call()
+    wb.record(s)
     torch.cuda.synchronize()
+    est_ms = max(wa.elapsed_time(wb) / max(args.warmup, 1), 1e-3)
+    soak_n = int(250.0 / est_ms) + 1  # >= 250 ms of the same launches before the timed steps
 
     def timed():
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
               for _ in range(args.steps)]
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
         sampler = ClockSampler(local_rank)
         with sampler:
+            for _ in range(soak_n):  # clock soak (untimed): the sampler sees a sustained load
+                call()
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            n_soak = len(sampler.samples)
             t0.record(s)
             for a, b in ev:
                 a.record(s)
@@ -304,6 +325,7 @@ def run_ours(args, workload, rank, world, local_rank):
                 b.record(s)
             t1.record(s)
             torch.cuda.synchronize()
+            sampler.timed_samples = len(sampler.samples) - n_soak
         if world > 1:
             dist.barrier()
         return t0.elapsed_time(t1), [a.elapsed_time(b) for a, b in ev], sampler
@@ -349,11 +371,15 @@ def run_ours(args, workload, rank, world, local_rank):
                "steps": e2e_steps, "path": "sat_compute_host (pinned host in/out, banded H2D/SAT/D2H overlap)"}
         del xh, oh
 
-    banded = None
-    if world > 1 or args.banded:
+    sharded = banded = None
+    if not args.no_extras:
+        try:
+            sharded = run_sharded_batch(args, rank, world, local_rank)
+        except Exception as ex:  # report it on the line; the headline above stands
+            sharded = {"workload": "batch-1024x1080x1920-8u32s", "error": str(ex)[:300]}
         try:
             banded = run_banded(args, rank, world, local_rank)
-        except Exception as ex:  # report it on the line; the headline above stands
+        except Exception as ex:
             banded = {"workload": "huge-65536sq-32f32f row-banded", "error": str(ex)[:300]}
 
     if rank != 0:
@@ -373,9 +399,14 @@ def run_ours(args, workload, rank, world, local_rank):
                      "algorithmic_bytes_per_launch": alg_bytes,
                      "kernel_ms_mean": kern_ms, "kernel_ms_min": min(per)},
         "gpu_launches": args.steps,
-        "clocks": sampler.summary() | {"remeasured": remeasured},
+        "clocks": sampler.summary() | {"remeasured": remeasured, "soak_launches": soak_n,
+                                        "soak_ms": round(soak_n * est_ms, 1),
+                                        "samples_in_timed_steps": getattr(sampler, "timed_samples", None),
+                                        "covers": "soak of the same launches + the timed steps"},
         "e2e": e2e,
     }
+    if sharded is not None:
+        line["sharded_batch"] = sharded
     if banded is not None:
         line["banded"] = banded
     if world == 1 and not args.no_sweep:
@@ -398,12 +429,76 @@ def run_ours(args, workload, rank, world, local_rank):
     print(json.dumps(line), flush=True)
 
 
+def _max_over_ranks(torch, dist, dev, world, ms):
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    return ms
+
+
+def _timed_ms(torch, dist, world, s, fn, steps):
+    """Mean device ms per call of fn(): barrier + sync, events on stream s."""
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(s)
+    for _ in range(steps):
+        fn()
+    b.record(s)
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / steps
+
+
+def run_sharded_batch(args, rank, world, local_rank, F=1024, H=1080, W=1920, seed=1002):
+    """BASELINE configs[2]: 1024 1080x1920 8u frames sharded by image: rank r
+    computes frames [r*F/P, (r+1)*F/P) with one sat_compute_batched per step
+    (no data-path collective).  Strong scaling: the total work is fixed."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cluster_chenwttm18_b200 as sat
+    import satgen
+
+    dev = torch.device("cuda", local_rank)
+    f0, f1 = rank * F // world, (rank + 1) * F // world
+    n = f1 - f0
+    x = torch.empty((n, H, W), dtype=torch.uint8, device=dev)
+    satgen.fill_device(x, seed=seed, img0=f0)
+    out = torch.empty((n, H, W), dtype=torch.int32, device=dev)
+    plan = sat.Plan(0, H, W, n, dev)
+    s = torch.cuda.current_stream(dev)
+    call = lambda: plan.compute_batched_ptr(x.data_ptr(), out.data_ptr(), H, W, W, W * 4, H * W,
+                                            H * W * 4, n, s)
+    for _ in range(max(3, args.warmup)):
+        call()
+    steps = max(3, min(args.steps, 10))
+    ms = _max_over_ranks(torch, dist, dev, world, _timed_ms(torch, dist, world, s, call, steps))
+    del x, out
+    plan.close()
+    torch.cuda.empty_cache()
+    px = F * H * W
+    return {"workload": "batch-1024x1080x1920-8u32s", "frames_per_rank": n, "n_gpus": world,
+            "steps": steps, "ms_per_step": ms, "value": px / (ms * 1e-3) / 1e9, "unit": "Gpx/s",
+            "scaling": "strong", "parallelism": f"frames sharded x{world}, no collective",
+            "rank_alg_gbs": n * H * W * 5 / (ms * 1e-3) / 1e9}
+
+
 def run_banded(args, rank, world, local_rank, H=65536, W=65536, pair=1, seed=1004):
     """BASELINE configs[3]: ONE 65536 x 65536 32f image row-banded across the
-    ranks (sat_compute_dist: band column sums -> ncclAllGather of the W-vectors
-    -> carry row -> band SAT with the carry fused).  Timed like the headline
-    (barrier + events on the launching stream, max over ranks); value = the
-    whole image's pixels / step time."""
+    ranks, both multi-GPU schemes, timed like the headline (barrier + events on
+    the launching stream, max over ranks); value = the whole image's pixels /
+    step time (strong scaling).
+      colsum  : sat_compute_dist (band column sums -> ncclAllGather of the
+                W-vectors -> carry row -> band SAT with the carry fused); its
+                phases are also timed one by one through the exported building
+                blocks (sat_dist_colsum, a torch NCCL all-gather of the same
+                vectors, sat_dist_carry, sat_compute_band);
+      chained : sat_compute_dist_chained (one kernel per rank; bottom rows
+                published into the next GPU's link over NVLink peer memory).
+    The two legs' outputs are compared (different algorithms; both must be
+    within the 1e-4 bar of the exact SAT, so they must agree within 2e-4)."""
     import torch
     import torch.distributed as dist
 
@@ -421,47 +516,87 @@ def run_banded(args, rank, world, local_rank, H=65536, W=65536, pair=1, seed=100
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
         own_pg = True
     r0, r1 = sat.band_partition(H, world, rank)
+    bh = r1 - r0
     dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64}[pair]
-    band = torch.empty((r1 - r0, W), dtype=dt, device=dev)
+    band = torch.empty((bh, W), dtype=dt, device=dev)
     satgen.fill_device(band, seed=seed, y0=r0)
-    out = torch.empty((r1 - r0, W), dtype=sat.out_dtype(pair), device=dev)
-    plan = sat.Plan(pair, max(r1 - r0, 1), W, 1, dev)
+    out_c = torch.empty((bh, W), dtype=sat.out_dtype(pair), device=dev)
+    out_x = torch.empty((bh, W), dtype=sat.out_dtype(pair), device=dev)
+    plan = sat.Plan(pair, bh, W, 1, dev)
     comm = sat.SatComm(device=dev)
     s = torch.cuda.current_stream(dev)
     steps = max(3, min(args.steps, 10))
+    res = {"workload": "huge-65536sq-32f32f row-banded", "n_gpus": world, "steps": steps,
+           "unit": "Gpx/s", "scaling": "strong", "rank0_band_rows": bh}
+    px = H * W
+    # -- colsum leg
+    col = lambda: sat.sat_dist(band, comm, out=out_c, plan=plan)
     for _ in range(max(3, args.warmup)):
-        sat.sat_dist(band, comm, out=out, plan=plan)
-    torch.cuda.synchronize()
+        col()
+    ms_c = _max_over_ranks(torch, dist, dev, world, _timed_ms(torch, dist, world, s, col, steps))
+    reads = 2 if world > 1 else 1
+    res["colsum"] = {"ms_per_step": ms_c, "value": px / (ms_c * 1e-3) / 1e9,
+                     "hbm_bytes_per_rank": bh * W * (reads * IN_B[pair] + OUT_B[pair])}
+    if world > 1:  # phase by phase (same kernels as sat_compute_dist)
+        acc_dt = torch.int32 if pair == 0 else torch.float64
+        acc = torch.empty(W, dtype=acc_dt, device=dev)
+        gathered = torch.empty((world, W), dtype=acc_dt, device=dev)
+        carry = torch.empty(W, dtype=sat.out_dtype(pair), device=dev)
+        phases = {
+            "colsum": lambda: sat.dist_colsum(band, plan=plan, pair=pair),
+            "allgather": lambda: dist.all_gather_into_tensor(gathered, acc),
+            "carry": lambda: sat.lib().sat_dist_carry(plan.handle, gathered.data_ptr(), world, rank, W,
+                                                      carry.data_ptr(), sat._stream_ptr(None, dev)),
+            "band_sat": lambda: sat.sat_band(band, carry_in=carry if rank > 0 else None, out=out_c,
+                                             plan=plan),
+        }
+        res["colsum"]["phase_ms"] = {}
+        for name, fn in phases.items():
+            fn()
+            res["colsum"]["phase_ms"][name] = _max_over_ranks(
+                torch, dist, dev, world, _timed_ms(torch, dist, world, s, fn, steps))
+        col()  # out_c = the full colsum-path result again
+    # -- chained leg
     if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    a.record(s)
-    for _ in range(steps):
-        sat.sat_dist(band, comm, out=out, plan=plan)
-    b.record(s)
-    torch.cuda.synchronize()
-    ms = a.elapsed_time(b) / steps
-    if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        ch = lambda: sat.sat_dist_chained(band, comm, out=out_x, plan=plan)
+        for _ in range(max(3, args.warmup)):
+            ch()
+        ms_x = _max_over_ranks(torch, dist, dev, world, _timed_ms(torch, dist, world, s, ch, steps))
+        plan.status()  # no bounded wait ran out
+        res["chained"] = {"ms_per_step": ms_x, "value": px / (ms_x * 1e-3) / 1e9,
+                          "hbm_bytes_per_rank": bh * W * (IN_B[pair] + OUT_B[pair]),
+                          "kernels_per_rank_per_step": 1}
+        torch.cuda.synchronize()
+        # cross-check of the two legs on this rank's band
+        if pair == 0:
+            agree = bool(torch.equal(out_c, out_x))
+            rel = 0.0 if agree else None
+        else:
+            rel = 0.0
+            for y0 in range(0, bh, 4096):  # chunked: bounded temporaries
+                a_ = out_c[y0:y0 + 4096].double()
+                b_ = out_x[y0:y0 + 4096].double()
+                rel = max(rel, float(((a_ - b_).abs() / a_.abs().clamp_min(1e-300)).max()))
+            agree = rel <= 2e-4
+        t = torch.tensor([0.0 if agree else 1.0, rel or 0.0], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
-        dist.barrier()
+        res["legs_agree"] = {"all_ranks": bool(t[0].item() == 0.0), "max_rel_diff": float(t[1].item()),
+                             "bar": "bit-exact (8u) / <= 2e-4 (both legs within 1e-4 of exact)"}
+        best = min(ms_c, ms_x)
+        res.update({"ms_per_step": best, "value": px / (best * 1e-3) / 1e9,
+                    "parallelism": f"row bands x{world}; value = faster leg"})
+    else:
+        res.update({"ms_per_step": ms_c, "value": res["colsum"]["value"],
+                    "parallelism": "one GPU: the whole image (no exchange)"})
     comm.close()
+    plan.close()
+    if world > 1:
+        dist.barrier()
     if own_pg:
         dist.destroy_process_group()
-    del band, out
+    del band, out_c, out_x
     torch.cuda.empty_cache()
-    px = H * W
-    # per rank: the band is read twice (column sums, then the SAT) and written
-    # once; a single rank has no carry to exchange (sat_compute_dist runs the SAT only)
-    reads = 2 if world > 1 else 1
-    per_rank_bytes = (r1 - r0) * W * (reads * IN_B[pair] + OUT_B[pair])
-    return {"workload": "huge-65536sq-32f32f row-banded", "n_gpus": world, "steps": steps,
-            "ms_per_step": ms, "value": px / (ms * 1e-3) / 1e9, "unit": "Gpx/s",
-            "scaling": "strong", "parallelism": f"row bands x{world} (ncclAllGather carry)",
-            "rank0_band_rows": r1 - r0, "hbm_bytes_per_rank": per_rank_bytes,
-            "rank_gbs": per_rank_bytes / (ms * 1e-3) / 1e9}
+    return res
 
 
 def main():
@@ -472,8 +607,8 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD, choices=sorted(WORKLOADS))
     ap.add_argument("--no-sweep", action="store_true")
-    ap.add_argument("--banded", action="store_true",
-                    help="also time the row-banded 65536^2 32f path (always on for N > 1)")
+    ap.add_argument("--no-extras", action="store_true",
+                    help="skip the sharded_batch and banded objects (configs[2], configs[3])")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))

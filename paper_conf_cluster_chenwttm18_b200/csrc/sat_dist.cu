@@ -198,19 +198,67 @@ __global__ void __launch_bounds__(kCarryThreads)
   if (tid == kCarryThreads - 1) tile_tot[blockIdx.x] = wsum[kCarryThreads / 32 - 1];
 }
 
+// Phase 2: exclusive scan of the CTA totals by ONE WARP (ntiles = W / 4096,
+// e.g. 16 at W = 65536): lane l sums a contiguous segment serially
+// (compensated for doubles), the 32 segment totals are scanned with
+// shuffles in double-double arithmetic (TwoSum), and each lane writes its
+// segment's exclusive offsets.
+__device__ __forceinline__ void two_sum(double a, double b, double& s, double& e) {
+  s = a + b;
+  const double bb = s - a;
+  e = (a - (s - bb)) + (b - bb);
+}
+
 template <typename ACC>
 __global__ void sat_carry_offsets_kernel(ACC* __restrict__ tile_tot, int64_t ntiles) {
-  if (threadIdx.x != 0) return;
-  ACC run = ACC(0), runc = ACC(0);
-  for (int64_t i = 0; i < ntiles; ++i) {
-    const ACC v = tile_tot[i];
-    tile_tot[i] = run + runc;  // exclusive
+  const int lane = threadIdx.x;
+  const int64_t per = (ntiles + 31) / 32;
+  const int64_t i0 = ntiles < lane * per ? ntiles : lane * per;
+  const int64_t i1 = ntiles < i0 + per ? ntiles : i0 + per;
+  ACC hi = ACC(0), lo = ACC(0);  // segment total (hi + lo)
+  for (int64_t i = i0; i < i1; ++i) {
     if constexpr (sizeof(ACC) == 8) {
-      const ACC t = run + v;
-      runc += (fabs(run) >= fabs(v)) ? ((run - t) + v) : ((v - t) + run);
-      run = t;
+      double s, e;
+      two_sum(hi, tile_tot[i], s, e);
+      hi = s;
+      lo += e;
     } else {
-      run += v;
+      hi += tile_tot[i];
+    }
+  }
+  // inclusive warp scan of (hi, lo)
+  ACC ih = hi, il = lo;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const ACC oh = __shfl_up_sync(0xffffffffu, ih, d), ol = __shfl_up_sync(0xffffffffu, il, d);
+    if (lane >= d) {
+      if constexpr (sizeof(ACC) == 8) {
+        double s, e;
+        two_sum(ih, oh, s, e);
+        ih = s;
+        il = il + ol + e;
+      } else {
+        ih += oh;
+      }
+    }
+  }
+  ACC rh = ih - hi, rl = il - lo;  // exclusive: running offset of this segment
+  if constexpr (sizeof(ACC) == 8) {
+    double s, e;  // (ih, il) - (hi, lo) exactly enough: re-split the high part
+    two_sum(ih, -hi, s, e);
+    rh = s;
+    rl = il - lo + e;
+  }
+  for (int64_t i = i0; i < i1; ++i) {
+    const ACC v = tile_tot[i];
+    tile_tot[i] = rh + rl;
+    if constexpr (sizeof(ACC) == 8) {
+      double s, e;
+      two_sum(rh, v, s, e);
+      rh = s;
+      rl += e;
+    } else {
+      rh += v;
     }
   }
 }
@@ -234,6 +282,8 @@ struct DistBufs {
   void* local = nullptr;     // [w] ACC
   void* gathered = nullptr;  // [nranks][w] ACC
   void* carry = nullptr;     // [w] TB
+  void* scratch = nullptr;   // band_carry scratch (zeroed once)
+  uint32_t epoch = 0;        // band_carry call counter (tile-flag epoch)
 };
 
 sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t pitch,
@@ -301,14 +351,122 @@ sat_status colsum(sat_pair pair, const void* in, int64_t h, int64_t w, int64_t p
   return e == cudaSuccess ? SAT_OK : cuda_fail(e, "sat_colsum_kernel launch");
 }
 
+// One-kernel carry row (ntiles <= kCarryFusedMaxTiles, all CTAs co-resident):
+// phase 1 as sat_carry_scan_kernel; each CTA publishes its tile total with an
+// epoch flag (release), warp 0 then sums the totals of the tiles to its left
+// (acquire; double-double for the float pairs, the same compensated sum as
+// the offsets kernel) and every thread adds that offset and rounds once to
+// T_B.  Same arithmetic as the three-kernel path, one launch instead of three.
+// Small tiles (1024 x) spread the gathered-vector reads over many CTAs.
+constexpr int kFusedThreads = 256;
+constexpr int64_t kFusedTile = kFusedThreads * kCarryItems;
+constexpr int64_t kCarryFusedMaxTiles = 512;  // <= co-resident 256-thread CTAs on 148 SMs
+
+template <typename ACC, typename TB>
+__global__ void __launch_bounds__(kFusedThreads)
+    sat_carry_fused_kernel(const ACC* __restrict__ gathered, int rank, int64_t w,
+                           TB* __restrict__ carry, ACC* tile_tot, uint32_t* flags, uint32_t epoch) {
+  __shared__ ACC wsum[32];
+  __shared__ ACC toff;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  constexpr int kW = kFusedThreads / 32;
+  const int64_t base = (int64_t)blockIdx.x * kFusedTile + (int64_t)tid * kCarryItems;
+  ACC v[kCarryItems];
+  ACC run = ACC(0);
+#pragma unroll
+  for (int k = 0; k < kCarryItems; ++k) {
+    const int64_t x = base + k;
+    ACC c = ACC(0);
+    if (x < w)
+      for (int r = 0; r < rank; ++r) c += gathered[(int64_t)r * w + x];
+    run += c;
+    v[k] = run;
+  }
+  const ACC incl = warp_incl_scan(run, lane);
+  if (lane == 31) wsum[wid] = incl;
+  __syncthreads();
+  if (wid == 0) {
+    const ACC ws = warp_incl_scan(lane < kW ? wsum[lane] : ACC(0), lane);
+    wsum[lane] = ws;
+  }
+  __syncthreads();
+  const ACC off = (incl - run) + (wid > 0 ? wsum[wid - 1] : ACC(0));
+  if (tid == 0) {
+    tile_tot[blockIdx.x] = wsum[kW - 1];
+    __threadfence();
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flags + blockIdx.x), "r"(epoch) : "memory");
+  }
+  if (wid == 0) {
+    ACC hi = ACC(0), lo = ACC(0);
+    for (int64_t i = lane; i < (int64_t)blockIdx.x; i += 32) {
+      uint32_t f;
+      do {
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(f) : "l"(flags + i) : "memory");
+      } while (f != epoch);
+      const ACC t = *reinterpret_cast<volatile ACC*>(tile_tot + i);
+      if constexpr (sizeof(ACC) == 8) {
+        double a, e;
+        two_sum(hi, t, a, e);
+        hi = a;
+        lo += e;
+      } else {
+        hi += t;
+      }
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+      const ACC oh = __shfl_down_sync(0xffffffffu, hi, d), ol = __shfl_down_sync(0xffffffffu, lo, d);
+      if constexpr (sizeof(ACC) == 8) {
+        double a, e;
+        two_sum(hi, oh, a, e);
+        hi = a;
+        lo = lo + ol + e;
+      } else {
+        hi += oh;
+      }
+    }
+    if (lane == 0) toff = hi + lo;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < kCarryItems; ++k)
+    if (base + k < w) carry[base + k] = (TB)(toff + (off + v[k]));
+}
+
+// Scratch of band_carry: local prefixes [w] + tile totals (8 bytes each) + tile flags.
+size_t carry_scratch_bytes(int64_t w) {
+  const int64_t nt = (w + kFusedTile - 1) / kFusedTile;  // >= the 3-kernel path's tile count
+  return (size_t)(w + nt) * 8 + (size_t)nt * 4;
+}
+
 sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, void* carry,
-                      cudaStream_t s) {
-  // scratch: local prefixes [w] + tile totals (stream-ordered allocation)
+                      void* scratch, uint32_t epoch, cudaStream_t s) {
   const int64_t ntiles = (w + kCarryTile - 1) / kCarryTile;
-  void* scratch = nullptr;
-  cudaError_t e = cudaMallocAsync(&scratch, (size_t)(w + ntiles) * 8, s);
-  if (e != cudaSuccess) return cuda_fail(e, "cudaMallocAsync(carry scratch)");
+  cudaError_t e = cudaSuccess;
   const unsigned fin = (unsigned)((w + 255) / 256);
+  const int64_t nfused = (w + kFusedTile - 1) / kFusedTile;
+  if (nfused <= kCarryFusedMaxTiles) {
+    const unsigned ntiles = (unsigned)nfused;
+    uint32_t* flags = reinterpret_cast<uint32_t*>(static_cast<char*>(scratch) + (size_t)(w + nfused) * 8);
+    switch (pair) {
+      case SAT_8U_32S:
+      case SAT_32S_32S:
+        sat_carry_fused_kernel<uint32_t, uint32_t><<<ntiles, kFusedThreads, 0, s>>>(
+            (const uint32_t*)gathered, rank, w, (uint32_t*)carry, (uint32_t*)scratch, flags, epoch);
+        break;
+      case SAT_32F_32F:
+      case SAT_8U_32F:
+        sat_carry_fused_kernel<double, float><<<ntiles, kFusedThreads, 0, s>>>(
+            (const double*)gathered, rank, w, (float*)carry, (double*)scratch, flags, epoch);
+        break;
+      case SAT_64F_64F:
+        sat_carry_fused_kernel<double, double><<<ntiles, kFusedThreads, 0, s>>>(
+            (const double*)gathered, rank, w, (double*)carry, (double*)scratch, flags, epoch);
+        break;
+    }
+    e = cudaGetLastError();
+    return e == cudaSuccess ? SAT_OK : cuda_fail(e, "sat_carry_fused_kernel launch");
+  }
   switch (pair) {
     case SAT_8U_32S:
     case SAT_32S_32S: {
@@ -334,7 +492,6 @@ sat_status band_carry(sat_pair pair, const void* gathered, int rank, int64_t w, 
     }
   }
   e = cudaGetLastError();
-  cudaFreeAsync(scratch, s);
   return e == cudaSuccess ? SAT_OK : cuda_fail(e, "carry kernels launch");
 }
 
@@ -376,6 +533,7 @@ static void free_bufs(DistBufs& b) {
   if (b.local) cudaFree(b.local);
   if (b.gathered) cudaFree(b.gathered);
   if (b.carry) cudaFree(b.carry);
+  if (b.scratch) cudaFree(b.scratch);
   b = DistBufs();
 }
 
@@ -389,6 +547,8 @@ static sat_status ensure_bufs(DistBufs& b, int64_t w, int nranks) {
   if (e == cudaSuccess) e = cudaMalloc(&b.local, (size_t)w * 8);
   if (e == cudaSuccess) e = cudaMalloc(&b.gathered, (size_t)nranks * w * 8);
   if (e == cudaSuccess) e = cudaMalloc(&b.carry, (size_t)w * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&b.scratch, carry_scratch_bytes(w));
+  if (e == cudaSuccess) e = cudaMemset(b.scratch, 0, carry_scratch_bytes(w));
   if (e != cudaSuccess) {
     free_bufs(b);
     return cuda_fail(e, "dist buffers");
@@ -452,6 +612,22 @@ sat_status sat_comm_destroy(sat_comm comm) {
   return SAT_OK;
 }
 
+// Plan-owned scratch of the exported building blocks: grown (synchronously,
+// after draining the plan's last stream) only when a wider call needs more.
+static sat_status plan_dist_scratch(sat_plan plan, size_t bytes) {
+  if (plan->dist_scratch_bytes >= bytes) return SAT_OK;
+  cudaDeviceSynchronize();
+  if (plan->dist_scratch) cudaFree(plan->dist_scratch);
+  plan->dist_scratch = nullptr;
+  plan->dist_scratch_bytes = 0;
+  cudaError_t e = cudaMalloc(&plan->dist_scratch, bytes);
+  if (e == cudaSuccess) e = cudaMemset(plan->dist_scratch, 0, bytes);
+  if (e != cudaSuccess) return cuda_fail(e, "dist scratch");
+  plan->dist_epoch = 0;
+  plan->dist_scratch_bytes = bytes;
+  return SAT_OK;
+}
+
 // Building blocks of sat_compute_dist, exported so that the carry algebra can
 // be exercised on one GPU with "virtual ranks" (tests/test_dist_gpu.py).
 size_t sat_dist_acc_bytes(sat_pair pair) { return acc_size(pair); }
@@ -465,13 +641,10 @@ sat_status sat_dist_colsum(sat_plan plan, const void* in_band, int64_t band_h, i
   if (in_pitch_bytes < w * (int64_t)in_size(plan->pair))
     return fail(SAT_ERR_INVALID_ARGUMENT, "bad pitch");
   DeviceGuard g(plan->device);
-  void* partial = nullptr;
-  cudaError_t e = cudaMallocAsync(&partial, (size_t)64 * w * 8, (cudaStream_t)stream);
-  if (e != cudaSuccess) return cuda_fail(e, "cudaMallocAsync");
-  sat_status st = colsum(plan->pair, in_band, band_h, w, in_pitch_bytes, partial, 64, acc_out,
-                         (cudaStream_t)stream);
-  cudaFreeAsync(partial, (cudaStream_t)stream);
-  return st;
+  sat_status st = plan_dist_scratch(plan, (size_t)64 * w * 8);
+  if (st != SAT_OK) return st;
+  return colsum(plan->pair, in_band, band_h, w, in_pitch_bytes, plan->dist_scratch, 64, acc_out,
+                (cudaStream_t)stream);
 }
 
 sat_status sat_dist_carry(sat_plan plan, const void* gathered, int nranks, int rank, int64_t w,
@@ -480,7 +653,11 @@ sat_status sat_dist_carry(sat_plan plan, const void* gathered, int nranks, int r
   if (nranks < 1 || rank < 0 || rank >= nranks || w <= 0)
     return fail(SAT_ERR_INVALID_ARGUMENT, "bad rank/extent");
   DeviceGuard g(plan->device);
-  return band_carry(plan->pair, gathered, rank, w, carry_out, (cudaStream_t)stream);
+  sat_status st = plan_dist_scratch(plan, carry_scratch_bytes(w));
+  if (st != SAT_OK) return st;
+  if (++plan->dist_epoch == 0) ++plan->dist_epoch;
+  return band_carry(plan->pair, gathered, rank, w, carry_out, plan->dist_scratch, plan->dist_epoch,
+                    (cudaStream_t)stream);
 }
 
 sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, void* out_band,
@@ -514,7 +691,8 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
   const ncclDataType_t dt = acc_size(pair) == 4 ? ncclUint32 : ncclFloat64;
   ncclResult_t r = nccl().AllGather(b.local, b.gathered, (size_t)w, dt, comm->comm, s);
   if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
-  st = band_carry(pair, b.gathered, comm->rank, w, b.carry, s);
+  if (++b.epoch == 0) ++b.epoch;  // tile flags: epoch-tagged, never re-zeroed
+  st = band_carry(pair, b.gathered, comm->rank, w, b.carry, b.scratch, b.epoch, s);
   if (st != SAT_OK) return st;
   if (band_h == 0) return SAT_OK;
   return launch(plan, in_band, out_band, band_h, w, in_pitch_bytes, out_pitch_bytes,

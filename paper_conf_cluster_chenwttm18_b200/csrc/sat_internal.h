@@ -43,6 +43,10 @@ struct sat_plan_st {
   cudaEvent_t last_ev = nullptr;
   cudaStream_t last_stream = nullptr;
   bool has_last = false;
+  // scratch of sat_dist_colsum / sat_dist_carry (lazily allocated, grown)
+  void* dist_scratch = nullptr;
+  size_t dist_scratch_bytes = 0;
+  uint32_t dist_epoch = 0;  // tile-flag epoch of the one-kernel carry
   // streamed host path (lazily allocated)
   sat::HostPath* host = nullptr;
 };

@@ -692,6 +692,7 @@ sat_status sat_plan_destroy(sat_plan plan) {
   cudaSetDevice(plan->device);
   host_path_release(plan);
   if (plan->ws) cudaFree(plan->ws);
+  if (plan->dist_scratch) cudaFree(plan->dist_scratch);
   if (plan->last_ev) cudaEventDestroy(plan->last_ev);
   cudaSetDevice(prev);
   delete plan;

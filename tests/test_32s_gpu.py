@@ -86,10 +86,10 @@ def test_32s_dist_virtual_ranks_and_chain():
         y = sat.sat_band(x[a:b], carry_in=carry if r > 0 else None)
         torch.cuda.synchronize()
         assert np.array_equal(y.cpu().numpy(), ref[a:b]), f"colsum rank {r}"
-    bufs = [sat.new_chain_buffer(sat.PAIR_32S_32S, W) for _ in range(P - 1)]
+    links = [sat.new_chain_buffer(sat.PAIR_32S_32S, W) for _ in range(P)]
     out = torch.empty((H, W), dtype=torch.int32, device="cuda")
     for r, (a, b) in enumerate(spans):
-        sat.sat_band_chained(x[a:b], bufs[r - 1] if r > 0 else None, bufs[r] if r < P - 1 else None, 1,
-                             out=out[a:b])
+        sat.sat_band_chained(x[a:b], links[r], links[r - 1] if r > 0 else None,
+                             links[r + 1] if r < P - 1 else None, 1, out=out[a:b])
     torch.cuda.synchronize()
     assert np.array_equal(out.cpu().numpy(), ref)

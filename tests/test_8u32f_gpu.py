@@ -130,11 +130,11 @@ def test_8u32f_dist_virtual_ranks_and_chain():
         y = sat.sat_band(x[a:b], carry_in=carry if r > 0 else None, out_dtype=torch.float32)
         torch.cuda.synchronize()
         assert _rel(y.cpu().numpy(), ref[a:b]) <= TOL, f"colsum rank {r}"
-    bufs = [sat.new_chain_buffer(3, W) for _ in range(P - 1)]
+    links = [sat.new_chain_buffer(3, W) for _ in range(P)]
     out = torch.empty((H, W), dtype=torch.float32, device="cuda")
     for r, (a, b) in enumerate(spans):
-        sat.sat_band_chained(x[a:b], bufs[r - 1] if r > 0 else None, bufs[r] if r < P - 1 else None, 1,
-                             out=out[a:b])
+        sat.sat_band_chained(x[a:b], links[r], links[r - 1] if r > 0 else None,
+                             links[r + 1] if r < P - 1 else None, 1, out=out[a:b])
     torch.cuda.synchronize()
     assert _rel(out.cpu().numpy(), ref) <= TOL
 

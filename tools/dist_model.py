@@ -59,10 +59,11 @@ def main():
     for P in Ps:
         spans = [sat.band_partition(H, P, r) for r in range(P)]
         gathered = torch.stack([sat.dist_colsum(x[a:b]) for a, b in spans])
-        bufs = [sat.new_chain_buffer(pair, W) for _ in range(P - 1)]
-        for r in range(P - 1):  # fill chain buffers once (epoch 1) so band r sees its carry
+        links = [sat.new_chain_buffer(pair, W) for _ in range(P)]
+        for r in range(P - 1):  # fill the links once (epoch 1) so band r sees its carry
             a, b = spans[r]
-            sat.sat_band_chained(x[a:b], bufs[r - 1] if r > 0 else None, bufs[r], 1, out=out[a:b])
+            sat.sat_band_chained(x[a:b], links[r], links[r - 1] if r > 0 else None, links[r + 1], 1,
+                                 out=out[a:b])
         colsum_ms, chained_ms = [], []
         for r, (a, b) in enumerate(spans):
             def colsum_rank():
@@ -71,8 +72,9 @@ def main():
                 sat.sat_band(x[a:b], carry_in=c if r > 0 else None, out=out[a:b])
 
             def chained_rank():
-                # chain_out is NOT written (None): only band r's own device work
-                sat.sat_band_chained(x[a:b], bufs[r - 1] if r > 0 else None, None, 1, out=out[a:b])
+                # the band below is NOT written (None): only band r's own device work
+                sat.sat_band_chained(x[a:b], links[r], links[r - 1] if r > 0 else None, None, 1,
+                                     out=out[a:b])
 
             colsum_ms.append(ev_time(colsum_rank))
             if r == P - 1:

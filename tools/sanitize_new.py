@@ -41,11 +41,12 @@ chk(np.allclose(sat.sat(xf).cpu().numpy(), oracle.sat(xf.cpu().numpy()), rtol=1e
 os.environ["SAT_SHORT"] = "0"
 # chained bands
 P, H, W = 3, 300, 517
-bufs = [sat.new_chain_buffer(0, W) for _ in range(P - 1)]
+links = [sat.new_chain_buffer(0, W) for _ in range(P)]
 out = torch.empty((H, W), dtype=torch.int32, device="cuda")
 for r in range(P):
     a, b = sat.band_partition(H, P, r)
-    sat.sat_band_chained(x8[a:b], bufs[r - 1] if r else None, bufs[r] if r < P - 1 else None, 1, out=out[a:b])
+    sat.sat_band_chained(x8[a:b], links[r], links[r - 1] if r else None,
+                         links[r + 1] if r < P - 1 else None, 1, out=out[a:b])
 chk(np.array_equal(out.cpu().numpy(), oracle.sat(A8)), "chained")
 # dist carry kernels (virtual ranks)
 spans = [sat.band_partition(H, P, r) for r in range(P)]
