@@ -223,3 +223,33 @@ def sat_32s(A: np.ndarray) -> np.ndarray:
     assert A.dtype == np.int32 and A.ndim == 2
     S = A.astype(np.int64).astype(np.uint64).cumsum(axis=0, dtype=np.uint64).cumsum(axis=1, dtype=np.uint64)
     return (S & np.uint64(0xFFFFFFFF)).astype(np.uint32).view(np.int32)
+
+
+# ---------------------------------------------------------------------------
+# Multi-channel consumers.  Both are Eq. 1
+# applied channel by channel to a per-pixel vector f(A):
+
+def sat_sq(A: np.ndarray):
+    """SAT and SAT of squares of a uint8 image (Viola-Jones variance
+    normalisation, PAPER.md:18-24 [2]): S = sum_{y<=i, x<=j} A(y, x) and
+    Q = sum_{y<=i, x<=j} A(y, x)^2, both exact and reported mod 2^32 as int32
+    (reading R2).  Returns an [..., H, W, 2] int32 array (S, Q interleaved).
+    Q reuses sat_32s on the squared image (squares <= 65025 fit int32)."""
+    assert A.dtype == np.uint8
+    if A.ndim == 3:
+        return np.stack([sat_sq(a) for a in A])
+    S = sat(np.ascontiguousarray(A))
+    Q = sat_32s(np.ascontiguousarray(A.astype(np.int32) ** 2))
+    return np.stack([S, Q], axis=-1)
+
+
+def integral_histogram(A: np.ndarray, bin_of: np.ndarray, nbins: int) -> np.ndarray:
+    """Integral histogram ([34], [38]): H_k(i, j) = number of
+    pixels (y <= i, x <= j) whose value falls in bin k, bin = bin_of[value],
+    for k < nbins; counts exact mod 2^32 as int32.  Returns [nbins, H, W]
+    (bin-major; the library's interleaved 4-bin groups are compared after a
+    transpose).  Each bin is the SAT (`sat`, the int64 recurrence) of its
+    0/1 indicator image."""
+    assert A.dtype == np.uint8 and A.ndim == 2
+    b = np.asarray(bin_of, dtype=np.int64)[A]
+    return np.stack([sat(np.ascontiguousarray((b == k).astype(np.uint8))) for k in range(nbins)])

@@ -56,3 +56,64 @@ def test_box_filter_bruteforce_and_identity():
         for x in range(10):
             s = int(A[max(y - 2, 0):y + 3, max(x - 1, 0):x + 2].astype(np.int64).sum())
             assert got[y, x] == s
+
+
+# ---------------------------------------------------------------------------
+# Multi-channel consumers: SAT + SAT of squares, integral histogram.
+
+def test_sat_sq_bruteforce():
+    """Direct rectangle sums of A and A^2 from the origin (Eq. 1 by its
+    definition), exact integers."""
+    A = RNG.integers(0, 256, (7, 11)).astype(np.uint8)
+    SQ = oracle.sat_sq(A)
+    for i in range(7):
+        for j in range(11):
+            blk = A[:i + 1, :j + 1].astype(np.int64)
+            assert SQ[i, j, 0] == blk.sum()
+            assert SQ[i, j, 1] == (blk * blk).sum()
+
+
+def test_sat_sq_closed_form_and_wrap():
+    """Constant c: S = c (i+1)(j+1), Q = c^2 (i+1)(j+1) mod 2^32 -- c = 255 on
+    300 x 300 pushes Q past 2^32 (5.85e9)."""
+    c = 255
+    A = np.full((300, 300), c, dtype=np.uint8)
+    SQ = oracle.sat_sq(A)
+    ii, jj = np.meshgrid(np.arange(1, 301, dtype=np.int64), np.arange(1, 301, dtype=np.int64),
+                         indexing="ij")
+    wrap = lambda v: (v & 0xFFFFFFFF).astype(np.uint32).view(np.int32)
+    assert np.array_equal(SQ[..., 0], wrap(c * ii * jj))
+    assert np.array_equal(SQ[..., 1], wrap(c * c * ii * jj))
+    assert int(SQ[..., 1].view(np.uint32).max()) < c * c * 300 * 300  # it did wrap
+
+
+def test_sat_sq_variance_identity():
+    """A window's variance from the four corners of S and Q equals
+    numpy's variance of the window (the Viola-Jones use)."""
+    A = RNG.integers(0, 256, (40, 50)).astype(np.uint8)
+    SQ = oracle.sat_sq(A).astype(np.int64)
+    Z = np.zeros((41, 51, 2), dtype=np.int64)
+    Z[1:, 1:] = SQ
+    for (y0, x0, y1, x1) in [(0, 0, 40, 50), (3, 4, 27, 30), (10, 10, 12, 11)]:
+        s, q = (Z[y1, x1] - Z[y0, x1] - Z[y1, x0] + Z[y0, x0])
+        n = (y1 - y0) * (x1 - x0)
+        var = q / n - (s / n) ** 2
+        assert abs(var - A[y0:y1, x0:x1].astype(np.float64).var()) < 1e-6
+
+
+def test_integral_histogram_bruteforce_and_partition():
+    """Counts by direct counting over the prefix rectangle; the bins of a
+    table that covers every value sum to (i+1)(j+1); a value mapped outside
+    [0, nbins) is in no bin."""
+    A = RNG.integers(0, 256, (6, 9)).astype(np.uint8)
+    bin_of = RNG.integers(0, 5, 256)
+    bin_of[7] = 200  # never counted
+    A[2, 3] = 7
+    Hh = oracle.integral_histogram(A, bin_of, 5)
+    for k in range(5):
+        for i in range(6):
+            for j in range(9):
+                assert Hh[k, i, j] == int(np.sum(bin_of[A[:i + 1, :j + 1]] == k))
+    full = oracle.integral_histogram(A, np.arange(256) * 16 // 256, 16)
+    ii, jj = np.meshgrid(np.arange(1, 7), np.arange(1, 10), indexing="ij")
+    assert np.array_equal(full.sum(axis=0), ii * jj)
