@@ -56,9 +56,10 @@ WORKLOADS = {
     "64f-16384sq": (2, 16384, 16384, 1, 1005),
 }
 DEFAULT_WORKLOAD = "sweep-16384sq-8u32s"
-PAIR_NAME = {0: "8u->32s", 1: "32f->32f", 2: "64f->64f", 3: "8u->32f", 4: "32s->32s"}
-IN_B = {0: 1, 1: 4, 2: 8, 3: 1, 4: 4}
-OUT_B = {0: 4, 1: 4, 2: 8, 3: 4, 4: 4}
+PAIR_NAME = {0: "8u->32s", 1: "32f->32f", 2: "64f->64f", 3: "8u->32f", 4: "32s->32s",
+             5: "8u->(S, S of squares) 2x32u", 6: "8u->4-bin integral histogram 4x32u"}
+IN_B = {0: 1, 1: 4, 2: 8, 3: 1, 4: 4, 5: 1, 6: 1}
+OUT_B = {0: 4, 1: 4, 2: 8, 3: 4, 4: 4, 5: 8, 6: 16}
 DTYPE_NAME = {0: "u32", 1: "f32", 2: "f64"}
 L2_BYTES = 126 * 1024 * 1024
 
@@ -224,13 +225,20 @@ def cpu_baseline(workload, budget_s=10.0):
             "host_cpu": model, "host_cores": ncpu}
 
 
-def time_device(sat, x, out, steps, warmup, flush=None, stream=None):
-    """Per-step CUDA-event durations (ms) of sat(x -> out) on `stream`."""
+def time_device(sat, x, out, steps, warmup, flush=None, stream=None, pair=None):
+    """Per-step CUDA-event durations (ms) of sat(x -> out) on `stream` (for the
+    multi-channel pairs: one sat_sq / one 4-bin integral-histogram launch)."""
     import torch
 
     s = stream or torch.cuda.current_stream()
+    if pair == 5:
+        fn = lambda: sat.sat_sq(x, out=out, stream=s)
+    elif pair == 6:
+        fn = lambda: sat.integral_histogram(x, bins=4, out=out, stream=s)
+    else:
+        fn = lambda: sat.sat(x, out=out, stream=s)
     for _ in range(warmup):
-        sat.sat(x, out=out, stream=s)
+        fn()
     torch.cuda.synchronize()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(steps)]
@@ -238,24 +246,26 @@ def time_device(sat, x, out, steps, warmup, flush=None, stream=None):
         if flush is not None:
             flush.zero_()
         a.record(s)
-        sat.sat(x, out=out, stream=s)
+        fn()
         b.record(s)
     torch.cuda.synchronize()
     return [a.elapsed_time(b) for a, b in ev]
 
 
 def sweep_entry(sat, satgen, torch, pair, H, W, N, seed, steps, peak):
-    dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64, 3: torch.uint8, 4: torch.int32}[pair]
+    dt = {0: torch.uint8, 1: torch.float32, 2: torch.float64, 3: torch.uint8, 4: torch.int32,
+          5: torch.uint8, 6: torch.uint8}[pair]
     shape = (N, H, W) if N > 1 else (H, W)
     x = torch.empty(shape, dtype=dt, device="cuda")
     if pair == 4:  # satgen has no int32 kind: full-range torch randoms (every sum wraps)
         x.random_(-2**31, 2**31 - 1, generator=torch.Generator(device="cuda").manual_seed(seed))
     else:
         satgen.fill_device(x, seed=seed)
-    out = torch.empty(shape, dtype=sat.out_dtype(pair), device="cuda")
+    oshape = {5: (*shape, 2), 6: (1, *shape, 4)}.get(pair, shape)
+    out = torch.empty(oshape, dtype=sat.out_dtype(pair), device="cuda")
     byts = H * W * N * (IN_B[pair] + OUT_B[pair])
     flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device="cuda") if byts < 4 * L2_BYTES else None
-    ts = time_device(sat, x, out, steps, 3, flush)
+    ts = time_device(sat, x, out, steps, 3, flush, pair=pair)
     ms = statistics.median(ts)
     l2 = "flushed" if flush is not None else "inputs > L2"
     del x, out, flush
@@ -416,7 +426,8 @@ def run_ours(args, workload, rank, world, local_rank):
                                  (1, 8192, 8192, 1), (1, 16384, 16384, 1), (2, 16384, 16384, 1),
                                  (2, 4096, 65536, 1), (2, 65536, 4096, 1), (0, 4096, 65536, 1),
                                  (1, 65536, 4096, 1), (0, 1080, 1920, 1024),
-                                 (1, 65536, 65536, 1), (3, 16384, 16384, 1), (4, 16384, 16384, 1)]:
+                                 (1, 65536, 65536, 1), (3, 16384, 16384, 1), (4, 16384, 16384, 1),
+                                 (5, 16384, 16384, 1), (6, 16384, 16384, 1), (5, 1080, 1920, 256)]:
             try:
                 sweep.append(sweep_entry(sat, satgen, torch, p_, h_, w_, n_, 1001, 10, peak))
             except Exception as ex:  # e.g. OOM: report, keep going

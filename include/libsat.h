@@ -74,7 +74,22 @@ typedef enum {
 /* Type pairs T_A -> T_B.  SAT_8U_32F is NPP's second pair
  * (nppiIntegral_8u32f): uint8 input, float output accumulated in
  * fp32 (tolerance 1e-4 relative to the exact sum, as for 32f). */
-typedef enum { SAT_8U_32S = 0, SAT_32F_32F = 1, SAT_64F_64F = 2, SAT_8U_32F = 3, SAT_32S_32S = 4 } sat_pair;
+/* Multi-channel pairs (SAT consumers that motivate the primitive):
+ *   SAT_8U_SQ    : uint8 -> 2 x uint32 per pixel, interleaved (S, Q): S = the SAT
+ *                  of A and Q = the SAT of A^2 (Viola-Jones variance
+ *                  normalisation [2]), both exact mod 2^32 (reading R2), from ONE
+ *                  read of A in ONE pass (1 + 8 bytes per pixel).  A rectangle sum
+ *                  by four corners is exact when its true value is below
+ *                  2^32: every window of A, and windows of A^2 up to 66051 pixels.
+ *   SAT_8U_HIST4 : uint8 -> 4 x uint32 per pixel, interleaved: the integral
+ *                  histogram ([34], [38]) of bins [bin0, bin0 + 4) for a byte-to-
+ *                  bin table (sat_compute_hist4), counts exact mod 2^32.
+ * Output pitches / strides are in bytes of these 8- / 16-byte elements.  These
+ * pairs support sat_compute / sat_compute_batched (and sat_compute_hist4) only. */
+typedef enum {
+  SAT_8U_32S = 0, SAT_32F_32F = 1, SAT_64F_64F = 2, SAT_8U_32F = 3, SAT_32S_32S = 4,
+  SAT_8U_SQ = 5, SAT_8U_HIST4 = 6
+} sat_pair;
 
 typedef struct sat_plan_st* sat_plan;
 typedef struct sat_comm_st* sat_comm;
@@ -118,6 +133,19 @@ sat_status sat_compute_batched(sat_plan plan, const void* in, void* out, int64_t
                                int64_t in_pitch_bytes, int64_t out_pitch_bytes,
                                int64_t in_image_stride_bytes, int64_t out_image_stride_bytes,
                                int64_t batch, sat_pair pair, void* stream);
+
+/* Integral histogram, four bins per call (SAT_8U_HIST4 plans; PAPER.md:22,
+ * [34], [38]): out(y, x, k) = #{ (y', x') : y' <= y, x' <= x,
+ * bin_of[A(y', x')] == bin0 + k } for k < 4, uint32, interleaved per pixel
+ * (16 bytes).  bin_of: 256 entries, HOST memory (copied into the launch);
+ * values outside [bin0, bin0 + 4) are not counted.  K bins = ceil(K / 4)
+ * calls, each one pass (1 + 16 bytes per pixel).  Batches as
+ * sat_compute_batched.  Errors as sat_compute_batched; INVALID_ARGUMENT for
+ * a NULL table or a plan of another pair. */
+sat_status sat_compute_hist4(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                             int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                             int64_t in_image_stride_bytes, int64_t out_image_stride_bytes,
+                             int64_t batch, const uint8_t* bin_of, int bin0, void* stream);
 
 /* SAT of a row band with a carry-in row: out(i, j) = carry_in[j] + S_band(i, j),
  * where carry_in (device, w elements of T_B, contiguous) is the SAT row just
@@ -171,14 +199,16 @@ sat_status sat_compute_exclusive(sat_plan plan, const void* in, void* out, int64
 /* n rectangle sums.  rects: device int32[n][4] = {y0, x0, y1, x1} (16-byte
  * aligned), the half-open rectangle [y0, y1) x [x0, x1) of the image;
  * coordinates are clamped to [0, h] / [0, w] and an empty rectangle sums to 0.
- * out: device T_B[n]. */
+ * out: device T_B[n]; for the multi-channel SATs (SAT_8U_SQ, SAT_8U_HIST4)
+ * uint32[n][K] (K = 2: sum of A, sum of A^2 -- a window's variance is
+ * Q/n - (S/n)^2; K = 4: the window's 4 bin counts). */
 sat_status sat_rect_sums(sat_plan plan, const void* sat, int64_t h, int64_t w,
                          int64_t sat_pitch_bytes, const void* rects, int64_t n, void* out,
                          sat_pair pair, void* stream);
 
 /* Box filter (box sum): out(y, x) = sum of A over [y-ry, y+ry] x [x-rx, x+rx]
  * clipped to the image, for every pixel; out is h x w of T_B (device, must not
- * overlap the SAT).  ry, rx >= 0. */
+ * overlap the SAT).  ry, rx >= 0.  Single-channel SATs only. */
 sat_status sat_box_filter(sat_plan plan, const void* sat, void* out, int64_t h, int64_t w,
                           int64_t sat_pitch_bytes, int64_t out_pitch_bytes, int64_t ry,
                           int64_t rx, sat_pair pair, void* stream);

@@ -26,11 +26,12 @@ import threading
 __all__ = ["SatError", "Plan", "sat", "sat_host", "sat_exclusive", "sat_band", "SatComm", "sat_dist",
            "sat_dist_chained", "sat_band_chained", "new_chain_buffer", "chain_bytes", "ChainLink",
            "PeerLink", "SatChain", "rect_sums",
-           "box_filter", "band_partition",
+           "box_filter", "band_partition", "sat_sq", "integral_histogram",
            "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "PAIR_8U_32F", "PAIR_32S_32S", "lib",
            "LIB_PATH"]
 
 PAIR_8U_32S, PAIR_32F_32F, PAIR_64F_64F, PAIR_8U_32F, PAIR_32S_32S = 0, 1, 2, 3, 4
+PAIR_8U_SQ, PAIR_8U_HIST4 = 5, 6  # multi-channel: (S, S of squares) / 4 histogram bins
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("SAT_LIBRARY") or os.path.join(_HERE, "libsat.so")
 COMM_ID_BYTES = 128
@@ -71,6 +72,7 @@ def lib():
                     "sat_compute_band": ([vp, vp, vp, i64, i64, i64, i64, vp, i32, vp], i32),
                     "sat_compute_host": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_exclusive": ([vp, vp, vp, i64, i64, i64, i64, i32, vp, i32, vp], i32),
+                    "sat_compute_hist4": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i64, vp, i32, vp], i32),
                     "sat_rect_sums": ([vp, vp, i64, i64, i64, vp, i64, vp, i32, vp], i32),
                     "sat_chain_bytes": ([i32, i64], sz),
                     "sat_compute_band_chained": ([vp, vp, vp, i64, i64, i64, i64, vp, vp, vp, ctypes.c_uint32, i32, vp], i32),
@@ -127,7 +129,8 @@ def pair_of_dtype(dtype, out=None) -> int:
 def out_dtype(pair: int):
     torch = _torch()
     return {PAIR_8U_32S: torch.int32, PAIR_32F_32F: torch.float32, PAIR_64F_64F: torch.float64,
-            PAIR_8U_32F: torch.float32, PAIR_32S_32S: torch.int32}[pair]
+            PAIR_8U_32F: torch.float32, PAIR_32S_32S: torch.int32, PAIR_8U_SQ: torch.int32,
+            PAIR_8U_HIST4: torch.int32}[pair]
 
 
 _out_dtype_of = out_dtype  # for functions whose `out_dtype` parameter shadows the helper
@@ -302,20 +305,83 @@ def sat_exclusive(x, full: bool = True, nval=0, out=None, plan: Plan | None = No
     return out
 
 
+def sat_sq(x, out=None, plan: Plan | None = None, stream=None):
+    """SAT and SAT of squares of a uint8 CUDA image [H, W] or batch [N, H, W]
+    in ONE pass (Viola-Jones variance normalisation, PAPER.md:18-24 [2]):
+    returns int32 [..., H, W, 2] = (S, Q), both exact mod 2^32."""
+    torch = _torch()
+    if x.dtype != torch.uint8 or not x.is_cuda:
+        raise ValueError("sat_sq() takes a uint8 CUDA tensor")
+    if out is None:
+        out = torch.empty((*x.shape, 2), dtype=torch.int32, device=x.device)
+    H, W = x.shape[-2], x.shape[-1]
+    N = x.shape[0] if x.dim() == 3 else 1
+    if H == 0 or W == 0 or N == 0:
+        return out
+    ip, iis = _row_layout(x)
+    op, ois = out.stride(-3) * 4, (out.stride(0) * 4 if x.dim() == 3 else H * out.stride(-3) * 4)
+    p = plan if plan is not None else _plan_for(x.device, PAIR_8U_SQ, H, W, N)
+    p.compute_batched_ptr(x.data_ptr(), out.data_ptr(), H, W, ip, op, iis if N > 1 else H * ip,
+                          ois, N, stream)
+    return out
+
+
+def integral_histogram(x, bins=16, bin_of=None, out=None, plan: Plan | None = None, stream=None):
+    """Integral histogram of a uint8 CUDA image [H, W] ([34], [38]):
+    K = `bins` bins, value v in bin bin_of[v] (default: K equal-width bins,
+    bin_of[v] = v * K // 256).  Returns int32 [ceil(K/4), H, W, 4]: bin
+    4 * g + c is out[g, ..., c] (interleaved 4-bin groups; one single-pass
+    launch per group)."""
+    import numpy as np
+    torch = _torch()
+    if x.dtype != torch.uint8 or not x.is_cuda or x.dim() != 2:
+        raise ValueError("integral_histogram() takes a 2-D uint8 CUDA tensor")
+    table = (np.arange(256) * bins // 256) if bin_of is None else np.asarray(bin_of)
+    if table.shape != (256,) or table.min() < 0 or table.max() > 255:
+        raise ValueError("bin_of must be 256 bin indices in [0, 255]")
+    lut = (ctypes.c_uint8 * 256)(*[int(v) for v in table])
+    ngroups = (bins + 3) // 4
+    H, W = x.shape
+    if out is None:
+        out = torch.empty((ngroups, H, W, 4), dtype=torch.int32, device=x.device)
+    if H == 0 or W == 0:
+        return out
+    ip = _row_layout(x)[0]
+    p = plan if plan is not None else _plan_for(x.device, PAIR_8U_HIST4, H, W, 1)
+    for g in range(ngroups):
+        o = out[g]
+        _check(lib().sat_compute_hist4(p.handle, x.data_ptr(), o.data_ptr(), H, W, ip,
+                                       o.stride(0) * 4, H * ip, H * o.stride(0) * 4, 1, lut, 4 * g,
+                                       _stream_ptr(stream, x.device)), "sat_compute_hist4")
+    return out
+
+
 def rect_sums(S, rects, plan: Plan | None = None, stream=None):
     """Sums of A over half-open rectangles [y0, y1) x [x0, x1) from its inclusive
-    SAT S (a CUDA tensor as returned by sat()); rects: int32 CUDA tensor [n, 4]
-    of (y0, x0, y1, x1), clamped to the image."""
+    SAT S (a CUDA tensor as returned by sat(), or by sat_sq() / one group of
+    integral_histogram() -- [H, W, K] -> [n, K] results); rects: int32 CUDA
+    tensor [n, 4] of (y0, x0, y1, x1), clamped to the image."""
     torch = _torch()
-    pair = {torch.int32: 0, torch.float32: 1, torch.float64: 2}[S.dtype]
-    H, W = S.shape
+    if S.dim() == 3:  # multi-channel SAT [H, W, K]
+        pair = {2: PAIR_8U_SQ, 4: PAIR_8U_HIST4}[S.shape[2]]
+        H, W = S.shape[0], S.shape[1]
+        oshape = lambda n: (n, S.shape[2])
+    else:
+        pair = {torch.int32: 0, torch.float32: 1, torch.float64: 2}[S.dtype]
+        H, W = S.shape
+        oshape = lambda n: (n,)
     rects = rects.to(device=S.device, dtype=torch.int32).contiguous()
     if rects.dim() != 2 or rects.shape[1] != 4:
         raise ValueError("rects must be [n, 4]")
-    out = torch.empty(rects.shape[0], dtype=S.dtype, device=S.device)
+    out = torch.empty(oshape(rects.shape[0]), dtype=S.dtype, device=S.device)
     if rects.shape[0] == 0:
         return out
-    sp = _row_layout(S)[0] if H > 0 and W > 0 else max(W, 1) * S.element_size()
+    if S.dim() == 3:
+        if S.stride(2) != 1 or S.stride(1) != S.shape[2]:
+            raise ValueError("a multi-channel SAT must have contiguous [W, K] rows")
+        sp = S.stride(0) * 4 if H > 0 and W > 0 else max(W, 1) * S.shape[2] * 4
+    else:
+        sp = _row_layout(S)[0] if H > 0 and W > 0 else max(W, 1) * S.element_size()
     p = plan if plan is not None else _plan_for(S.device, pair, max(H, 1), max(W, 1), 1)
     _check(lib().sat_rect_sums(p.handle, S.data_ptr() if S.numel() else None, H, W, sp,
                                rects.data_ptr(), rects.shape[0], out.data_ptr(), pair,

@@ -634,6 +634,8 @@ size_t sat_dist_acc_bytes(sat_pair pair) { return acc_size(pair); }
 
 sat_status sat_dist_colsum(sat_plan plan, const void* in_band, int64_t band_h, int64_t w,
                            int64_t in_pitch_bytes, void* acc_out, void* stream) {
+  if (plan && multi_channel(plan->pair))
+    return fail(SAT_ERR_UNSUPPORTED, "row-banded building blocks: single-channel pairs only");
   if (!plan || !acc_out || (band_h > 0 && !in_band))
     return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
   if (band_h < 0 || w <= 0 || w > plan->max_w)
@@ -649,6 +651,8 @@ sat_status sat_dist_colsum(sat_plan plan, const void* in_band, int64_t band_h, i
 
 sat_status sat_dist_carry(sat_plan plan, const void* gathered, int nranks, int rank, int64_t w,
                           void* carry_out, void* stream) {
+  if (plan && multi_channel(plan->pair))
+    return fail(SAT_ERR_UNSUPPORTED, "row-banded building blocks: single-channel pairs only");
   if (!plan || !gathered || !carry_out) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL argument");
   if (nranks < 1 || rank < 0 || rank >= nranks || w <= 0)
     return fail(SAT_ERR_INVALID_ARGUMENT, "bad rank/extent");
@@ -665,6 +669,8 @@ sat_status sat_compute_dist(sat_plan plan, sat_comm comm, const void* in_band, v
                             int64_t out_pitch_bytes, sat_pair pair, void* stream) {
   if (!comm) return fail(SAT_ERR_INVALID_ARGUMENT, "comm is NULL");
   if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (multi_channel(plan->pair))
+    return fail(SAT_ERR_UNSUPPORTED, "row-banded SAT: single-channel pairs only");
   if (w <= 0) return fail(SAT_ERR_INVALID_ARGUMENT, "w must be positive for a collective call");
   bool empty = false;
   if (band_h > 0) {

@@ -16,8 +16,8 @@ struct sat_plan_st {
   sat_pair pair = SAT_8U_32S;
   int64_t max_h = 0, max_w = 0, max_batch = 0;
   int num_sms = 0;
-  int active_clusters[5][3][4] = {};  // [pair][cluster 2/4/8][mode: bit0 TMA, bit1 vec out]
-  int active_short[5] = {};           // [pair] short-band variant, clusters of 4, TMA + vec out
+  int active_clusters[7][3][4] = {};  // [pair][cluster 2/4/8][mode: bit0 TMA, bit1 vec out]
+  int active_short[7] = {};           // [pair] short-band variant, clusters of 4, TMA + vec out
   // Tuning / diagnosis knobs, read from the environment ONCE at plan creation
   // (SAT_FORCE_GENERIC, SAT_CLUSTER, SAT_SHORT, SAT_MAX_CLUSTERS,
   // SAT_FORCE_CLUSTERS, SAT_LOG); launches never consult the environment.
@@ -81,9 +81,16 @@ struct ChainSpec {
   const uint32_t* ack_in;  // this band's ack words (read before writing `out`)
   uint32_t epoch;
 };
+// Integral histogram (SAT_8U_HIST4): bin of every byte value, first bin of this launch.
+struct HistSpec {
+  const uint8_t* bin_of;  // 256 entries (host)
+  int bin0;
+};
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
-                  cudaStream_t stream, const ExSpec* ex = nullptr, const ChainSpec* chain = nullptr);
+                  cudaStream_t stream, const ExSpec* ex = nullptr, const ChainSpec* chain = nullptr,
+                  const HistSpec* hist = nullptr);
+bool multi_channel(sat_pair p);
 void host_path_release(sat_plan_st* pl);
 
 struct DeviceGuard {

@@ -69,15 +69,24 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <type_traits>
+
 namespace sat {
 
-enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2, P8U32F = 3, P32S32S = 4 };
+// P8USQ: 8u -> (S, S of squares), both u32 mod 2^32, interleaved per pixel
+// (Viola-Jones variance normalisation); P8UHIST4: 8u -> 4 bins of an integral
+// histogram (counts u32), interleaved per pixel.  Both are SATs of a per-pixel
+// vector f(a) (Eq. 1 applied channel by channel) on the same single pass.
+enum Pair : int { P8U32S = 0, P32F32F = 1, P64F64F = 2, P8U32F = 3, P32S32S = 4, P8USQ = 5,
+                  P8UHIST4 = 6 };
 // Short-band variants (P + kShort): the same pair with 16-row bands (2 rows per
 // compute warp), chosen for short, wide images whose 32-row bands would leave
 // most of the machine idle (H / 4 compute warps in total otherwise).
-constexpr int kShort = 5;
+constexpr int kShort = 8;
 template <int P>
 constexpr int kBase = P % kShort;
+template <int P>
+struct Cfg;
 
 #ifndef SAT_NLW
 #define SAT_NLW 1
@@ -157,6 +166,71 @@ struct Cfg<P32S32S> : Cfg<P32F32F> {
   using TB = uint32_t;
 };
 
+// K-channel u32 element (wrap-around adds per channel, exact mod 2^32).
+template <int K>
+struct ChanVec {
+  uint32_t c[K];
+  __device__ __forceinline__ ChanVec() {}
+  __device__ __forceinline__ ChanVec(int z) {
+#pragma unroll
+    for (int k = 0; k < K; ++k) c[k] = (uint32_t)z;
+  }
+  __device__ __forceinline__ ChanVec& operator+=(const ChanVec& o) {
+#pragma unroll
+    for (int k = 0; k < K; ++k) c[k] += o.c[k];
+    return *this;
+  }
+  __device__ __forceinline__ ChanVec operator+(const ChanVec& o) const {
+    ChanVec r = *this;
+    r += o;
+    return r;
+  }
+};
+template <int K>
+__device__ __forceinline__ ChanVec<K> shfl_up(const ChanVec<K>& v, int d) {
+  ChanVec<K> r;
+#pragma unroll
+  for (int k = 0; k < K; ++k) r.c[k] = __shfl_up_sync(0xffffffffu, v.c[k], d);
+  return r;
+}
+template <int K>
+__device__ __forceinline__ ChanVec<K> shfl_idx(const ChanVec<K>& v, int l) {
+  ChanVec<K> r;
+#pragma unroll
+  for (int k = 0; k < K; ++k) r.c[k] = __shfl_sync(0xffffffffu, v.c[k], l);
+  return r;
+}
+// 8u -> (a, a^2): 128-column tiles, a lane owns two groups of 2 pixels (16 B out each).
+template <>
+struct Cfg<P8USQ> {
+  using TA = uint8_t;
+  using TB = ChanVec<2>;
+  static constexpr int K = 2;
+  static constexpr int E = 2;
+  static constexpr int G = 2;
+  static constexpr int TW = 32 * E * G;  // 128
+  static constexpr int LOOK = 3;
+  static constexpr int NCW = 8;
+  static constexpr int TH = 32;
+  static constexpr int NSTAGE = 4;
+};
+// 8u -> 4 histogram bins: 64-column tiles, a lane owns two groups of 1 pixel.
+template <>
+struct Cfg<P8UHIST4> {
+  using TA = uint8_t;
+  using TB = ChanVec<4>;
+  static constexpr int K = 4;
+  static constexpr int E = 1;
+  static constexpr int G = 2;
+  static constexpr int TW = 32 * E * G;  // 64
+  static constexpr int LOOK = 3;
+  static constexpr int NCW = 8;
+  static constexpr int TH = 32;
+  static constexpr int NSTAGE = 4;
+};
+template <int P>
+constexpr bool kChan = kBase<P> == P8USQ || kBase<P> == P8UHIST4;
+
 template <int P>
 struct CfgShort : Cfg<P> {
   static constexpr int TH = Cfg<P>::TH / 2;
@@ -227,6 +301,8 @@ static_assert(kTmemColsPerSlot<P32F32F> * kNTot<P32F32F> <= kTmemCols<P32F32F>, 
 static_assert(kTmemColsPerSlot<P64F64F> * kNTot<P64F64F> <= kTmemCols<P64F64F>, "TMEM budget (64f)");
 static_assert(kTmemColsPerSlot<P8U32F> * kNTot<P8U32F> <= kTmemCols<P8U32F>, "TMEM budget (8u32f)");
 static_assert(kTmemColsPerSlot<P32S32S> * kNTot<P32S32S> <= kTmemCols<P32S32S>, "TMEM budget (32s)");
+static_assert(kTmemColsPerSlot<P8USQ> * kNTot<P8USQ> <= kTmemCols<P8USQ>, "TMEM budget (8u sq)");
+static_assert(kTmemColsPerSlot<P8UHIST4> * kNTot<P8UHIST4> <= kTmemCols<P8UHIST4>, "TMEM budget (hist)");
 
 struct KParams {
   const char* in;       // generic-path input base (TMA path uses the tensor map)
@@ -266,6 +342,10 @@ struct KParams {
   // reports SAT_ERR_TIMEOUT) instead of hanging the GPU.
   uint32_t* err;
   uint64_t spin_ns;
+  // Integral histogram (P8UHIST4): bin of every byte value; this launch
+  // counts bins [bin0, bin0 + 4).
+  uint8_t bin_of[256];
+  int32_t bin0;
 };
 
 // Optional phase profiling (debug builds with -DSAT_PROFILE): per-CTA shared
@@ -363,6 +443,8 @@ struct __align__(128) Smem {
   int32_t tot_k[kNTot<P>];
   int32_t tot_chunk[kNTot<P>];
   volatile uint32_t passA_done;                 // chunks through pass A (ticket pacing)
+  uint8_t bin_of[256];                          // P8UHIST4: byte -> bin (from KParams, in smem:
+                                                // divergent constant-bank reads serialise)
 #ifdef SAT_PROFILE
   unsigned long long prof[16];
 #endif
@@ -601,9 +683,16 @@ __device__ __forceinline__ void tmem_wait_ld() {
 // Pack / unpack a lane's RW x G x E values as 32-bit words for TMEM.
 __device__ __forceinline__ uint32_t w_lo(uint32_t v) { return v; }
 __device__ __forceinline__ uint32_t w_lo(float v) { return __float_as_uint(v); }
+template <typename T>
+struct IsChan : std::false_type {};
+template <int K>
+struct IsChan<ChanVec<K>> : std::true_type {};
 template <typename TB, int N>
 __device__ __forceinline__ void put_words(uint32_t (&w)[N], int idx, TB v) {
-  if constexpr (sizeof(TB) == 8) {
+  if constexpr (IsChan<TB>::value) {
+#pragma unroll
+    for (int k = 0; k < (int)(sizeof(TB) / 4); ++k) w[idx * (int)(sizeof(TB) / 4) + k] = v.c[k];
+  } else if constexpr (sizeof(TB) == 8) {
     const uint64_t b = (uint64_t)__double_as_longlong(v);
     w[2 * idx] = (uint32_t)b;
     w[2 * idx + 1] = (uint32_t)(b >> 32);
@@ -613,7 +702,12 @@ __device__ __forceinline__ void put_words(uint32_t (&w)[N], int idx, TB v) {
 }
 template <typename TB, int N>
 __device__ __forceinline__ TB get_words(const uint32_t (&w)[N], int idx) {
-  if constexpr (sizeof(TB) == 8) {
+  if constexpr (IsChan<TB>::value) {
+    TB v;
+#pragma unroll
+    for (int k = 0; k < (int)(sizeof(TB) / 4); ++k) v.c[k] = w[idx * (int)(sizeof(TB) / 4) + k];
+    return v;
+  } else if constexpr (sizeof(TB) == 8) {
     return __longlong_as_double((long long)(((uint64_t)w[2 * idx + 1] << 32) | w[2 * idx]));
   } else if constexpr (sizeof(TB) == 4 && TB(0.5) != TB(0)) {
     return __uint_as_float(w[idx]);
@@ -827,6 +921,153 @@ __device__ __forceinline__ void rows_scan(const double* tile, int lane, double (
   }
 }
 
+// Multi-channel pairs: a per-pixel vector f(a) whose channel-wise SAT is the
+// output (Eq. 1 per channel).  P8USQ: f(a) = (a, a^2) -- the SAT and the SAT
+// of squares of Viola-Jones variance normalisation ([2]);
+// P8UHIST4: f(a) = the indicator vector of bins [bin0, bin0 + 4) -- the
+// integral histogram ([34], [38]).
+template <int P>
+struct Xf;
+template <>
+struct Xf<P8USQ> {
+  static __device__ __forceinline__ ChanVec<2> f(uint32_t a, const KParams&) {
+    ChanVec<2> r;
+    r.c[0] = a;
+    r.c[1] = a * a;
+    return r;
+  }
+};
+template <>
+struct Xf<P8UHIST4> {
+  static __device__ __forceinline__ ChanVec<4> f(uint32_t a, const KParams& p) {
+    const int b = (int)p.bin_of[a] - p.bin0;
+    ChanVec<4> r;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) r.c[k] = b == k ? 1u : 0u;
+    return r;
+  }
+};
+
+// The lane's E consecutive bytes of group g of a tile row.
+template <int E>
+__device__ __forceinline__ uint32_t lane_bytes(const uint8_t* row, int col) {
+  if constexpr (E == 2) return *reinterpret_cast<const uint16_t*>(row + col);
+  else return row[col];
+}
+
+// a2 + a3 for the multi-channel pairs: per-lane serial prefix of the E pixels
+// of each group (Alg. 2), Kogge-Stone over the lanes (Alg. 3, lane >= d).
+template <int P, int RW>
+__device__ __forceinline__ void rows_scan_xf(const uint8_t* tile, int lane, const KParams& p,
+                                             typename Cfg<P>::TB (&rowcarry)[RW],
+                                             typename Cfg<P>::TB (&R)[RW][Cfg<P>::G][Cfg<P>::E]);
+
+// Integral histogram: a pixel's 4 bin indicators packed as 8-bit lanes of one
+// word (a tile row's prefix counts are <= 64), so the lane scan is ONE
+// Kogge-Stone on u32 words; unpacked onto the u32 row carries at the end.
+__device__ __forceinline__ uint32_t hist_pack(uint32_t a, const uint8_t* bin_of, int bin0) {
+  const int b = (int)bin_of[a] - bin0;
+  return (b >= 0 && b < 4) ? 1u << (8 * b) : 0u;
+}
+
+template <int RW>
+__device__ __forceinline__ void rows_scan_hist4(const uint8_t* tile, int lane, const uint8_t* lut,
+                                                int bin0, ChanVec<4> (&rowcarry)[RW],
+                                                ChanVec<4> (&R)[RW][2][1]) {
+  constexpr int TW = Cfg<P8UHIST4>::TW;  // 64: lane owns columns l and 32 + l
+  uint32_t own[RW][2], inc[RW][2];
+#pragma unroll
+  for (int i = 0; i < RW; ++i)
+#pragma unroll
+    for (int g = 0; g < 2; ++g) inc[i][g] = own[i][g] = hist_pack(tile[i * TW + g * 32 + lane], lut, bin0);
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    uint32_t o[RW][2];
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+#pragma unroll
+      for (int g = 0; g < 2; ++g) o[i][g] = __shfl_up_sync(kFull, inc[i][g], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+#pragma unroll
+      for (int g = 0; g < 2; ++g)
+        if (lane >= d) inc[i][g] += o[i][g];
+  }
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const uint32_t t0 = __shfl_sync(kFull, inc[i][0], 31), t1 = __shfl_sync(kFull, inc[i][1], 31);
+    const uint32_t p0 = inc[i][0], p1 = t0 + inc[i][1];  // inclusive prefixes, packed (<= 64 each)
+    const uint32_t tt = t0 + t1;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      R[i][0][0].c[k] = rowcarry[i].c[k] + ((p0 >> (8 * k)) & 0xffu);
+      R[i][1][0].c[k] = rowcarry[i].c[k] + ((p1 >> (8 * k)) & 0xffu);
+      rowcarry[i].c[k] += (tt >> (8 * k)) & 0xffu;
+    }
+  }
+}
+
+template <int P, int RW>
+__device__ __forceinline__ void rows_scan_chan(const uint8_t* tile, int lane, const KParams& p,
+                                               const uint8_t* lut,
+                                               typename Cfg<P>::TB (&rowcarry)[RW],
+                                               typename Cfg<P>::TB (&R)[RW][Cfg<P>::G][Cfg<P>::E]) {
+  if constexpr (P == P8UHIST4) {
+    rows_scan_hist4<RW>(tile, lane, lut, p.bin0, rowcarry, R);
+  } else {
+    rows_scan_xf<P, RW>(tile, lane, p, rowcarry, R);
+  }
+}
+
+template <int P, int RW>
+__device__ __forceinline__ void rows_scan_xf(const uint8_t* tile, int lane, const KParams& p,
+                                             typename Cfg<P>::TB (&rowcarry)[RW],
+                                             typename Cfg<P>::TB (&R)[RW][Cfg<P>::G][Cfg<P>::E]) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  TB inc[RW][C::G];  // R first holds the in-lane prefixes, then gets the bases added
+#pragma unroll
+  for (int i = 0; i < RW; ++i)
+#pragma unroll
+    for (int g = 0; g < C::G; ++g) {
+      const uint32_t b = lane_bytes<C::E>(tile + i * C::TW, g * 32 * C::E + lane * C::E);
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) {
+        const TB v = Xf<P>::f((b >> (8 * e)) & 0xffu, p);
+        R[i][g][e] = e == 0 ? v : R[i][g][e - 1] + v;
+      }
+      inc[i][g] = R[i][g][C::E - 1];
+    }
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    TB o[RW][C::G];
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+#pragma unroll
+      for (int g = 0; g < C::G; ++g) o[i][g] = shfl_up(inc[i][g], d);
+#pragma unroll
+    for (int i = 0; i < RW; ++i)
+#pragma unroll
+      for (int g = 0; g < C::G; ++g)
+        if (lane >= d) inc[i][g] += o[i][g];
+  }
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    TB base = rowcarry[i];
+#pragma unroll
+    for (int g = 0; g < C::G; ++g) {
+      const TB tot = shfl_idx(inc[i][g], 31);
+      TB ex = shfl_up(inc[i][g], 1);
+      if (lane == 0) ex = TB(0);
+      const TB bx = base + ex;
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) R[i][g][e] = bx + R[i][g][e];
+      base += tot;
+    }
+    rowcarry[i] = base;
+  }
+}
+
 // Carry payloads are epoch-TAGGED 64-bit words: (epoch << 32) | 32 value bits
 // (an fp64 value takes two words, low then high half).  A 64-bit store is
 // single-copy atomic, so a reader that sees the current epoch in a word also
@@ -861,6 +1102,26 @@ template <>
 struct Tag<P8U32F> : Tag<P32F32F> {};
 template <>
 struct Tag<P32S32S> : Tag<P8U32S> {};
+// K-channel elements: a 16-byte group is 4 u32 words whatever K is.
+template <int K, int E>
+struct TagChan {
+  static __device__ __forceinline__ void enc(const ChanVec<K> (&v)[E], uint32_t t, uint64_t (&w)[4]) {
+    uint32_t u[4];
+    memcpy(u, v, 16);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) w[e] = ((uint64_t)t << 32) | u[e];
+  }
+  static __device__ __forceinline__ void dec(const uint64_t (&w)[4], ChanVec<K> (&v)[E]) {
+    uint32_t u[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) u[e] = (uint32_t)w[e];
+    memcpy(v, u, 16);
+  }
+};
+template <>
+struct Tag<P8USQ> : TagChan<2, 2> {};
+template <>
+struct Tag<P8UHIST4> : TagChan<4, 1> {};
 template <>
 struct Tag<P64F64F> {
   static __device__ __forceinline__ void enc(const double (&v)[2], uint32_t t, uint64_t (&w)[4]) {
@@ -1376,7 +1637,11 @@ template <typename T>
 __device__ __forceinline__ T warp_incl(T v, int lane) {
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
-    const T o = __shfl_up_sync(kFull, v, d);
+    T o;
+    if constexpr (IsChan<T>::value)
+      o = shfl_up(v, d);
+    else
+      o = __shfl_up_sync(kFull, v, d);
     if (lane >= d) v += o;
   }
   return v;
@@ -1494,13 +1759,71 @@ struct Agg<P64F64F> {
   }
 };
 
+template <int P>
+struct AggChan {
+  using TB = typename Cfg<P>::TB;
+  using Acc = TB;
+  template <int TH>
+  static __device__ __forceinline__ void run(const uint8_t* tile, int lane, Acc& L,
+                                             TB (&agg)[Cfg<P>::G][Cfg<P>::E], const KParams& p,
+                                             const uint8_t* lut) {
+    using C = Cfg<P>;
+    TB c[C::G][C::E];
+    if constexpr (P == P8UHIST4) {  // column counts <= TH < 256: packed 8-bit lanes
+      static_assert(TH < 256, "packed histogram column counts");
+      uint32_t pk[2] = {0u, 0u};
+#pragma unroll 8
+      for (int r = 0; r < TH; ++r)
+#pragma unroll
+        for (int g = 0; g < 2; ++g) pk[g] += hist_pack(tile[r * C::TW + g * 32 + lane], lut, p.bin0);
+#pragma unroll
+      for (int g = 0; g < 2; ++g)
+#pragma unroll
+        for (int k = 0; k < 4; ++k) c[g][0].c[k] = (pk[g] >> (8 * k)) & 0xffu;
+    } else {
+#pragma unroll
+      for (int g = 0; g < C::G; ++g)
+#pragma unroll
+        for (int e = 0; e < C::E; ++e) c[g][e] = TB(0);
+#pragma unroll 4
+      for (int r = 0; r < TH; ++r)
+#pragma unroll
+        for (int g = 0; g < C::G; ++g) {
+          const uint32_t b = lane_bytes<C::E>(tile + r * C::TW, g * 32 * C::E + lane * C::E);
+#pragma unroll
+          for (int e = 0; e < C::E; ++e) c[g][e] += Xf<P>::f((b >> (8 * e)) & 0xffu, p);
+        }
+    }
+    TB base = L;
+#pragma unroll
+    for (int g = 0; g < C::G; ++g) {
+      TB pg[C::E];
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) pg[e] = e == 0 ? c[g][0] : pg[e - 1] + c[g][e];
+      const TB inc = warp_incl(pg[C::E - 1], lane);
+      const TB tot = shfl_idx(inc, 31);
+      TB ex = shfl_up(inc, 1);
+      if (lane == 0) ex = TB(0);
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) agg[g][e] = (base + ex) + pg[e];
+      base += tot;
+    }
+    L = base;
+  }
+};
+template <>
+struct Agg<P8USQ> : AggChan<P8USQ> {};
+template <>
+struct Agg<P8UHIST4> : AggChan<P8UHIST4> {};
+
 // Aggregate step (stage of chunk q landed): the band aggregate of the tile ->
 // the chunk's leader.  Returns false at the end-of-work sentinel, after giving
 // every leader warp of this CTA a sentinel in the gather slot of the next
 // chunk it would lead (its peers send nothing there).
 template <int P, int CL>
-__device__ __forceinline__ bool aggregate_step(Smem<P, CL>& sm, uint32_t rank, uint32_t q,
-                                               typename Agg<kBase<P>>::Acc& L, int lane) {
+__device__ __forceinline__ bool aggregate_step(Smem<P, CL>& sm, const KParams& p, uint32_t rank,
+                                               uint32_t q, typename Agg<kBase<P>>::Acc& L,
+                                               int lane) {
   using C = Cfg<P>;
   using TB = typename C::TB;
   using A = Agg<kBase<P>>;
@@ -1523,7 +1846,10 @@ __device__ __forceinline__ bool aggregate_step(Smem<P, CL>& sm, uint32_t rank, u
   const int32_t chunk = sm.stage_chunk[s];
   TB agg[C::G][C::E];
   if (chunk == 0) L = typename A::Acc(0);
-  A::template run<C::TH>(&sm.in[s][0][0], lane, L, agg);
+  if constexpr (kChan<P>)
+    A::template run<C::TH>(&sm.in[s][0][0], lane, L, agg, p, sm.bin_of);
+  else
+    A::template run<C::TH>(&sm.in[s][0][0], lane, L, agg);
   if (sm.stage_img[s] < 0) {  // padding band of a partial cluster: stage not loaded
 #pragma unroll
     for (int g = 0; g < C::G; ++g)
@@ -1574,7 +1900,8 @@ __device__ __forceinline__ uint32_t tmem_addr(const Smem<P, CL>& sm, int t, int 
 // tot[q % NT][warp]; the input stage is released at once.  Returns false at
 // the end-of-work sentinel.
 template <int P, int CL>
-__device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint32_t ph,
+__device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, const KParams& p, uint32_t q, int s,
+                                       uint32_t ph,
                                        typename Cfg<P>::TB (&rowcarry)[Cfg<P>::TH / kNCW<P>],
                                        int warp, int lane) {
   using C = Cfg<P>;
@@ -1596,7 +1923,10 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, uint32_t q, int s, uint3
   }
   const typename C::TA* tile = &sm.in[s][warp * RW][0];
   TB R[RW][C::G][C::E];
-  rows_scan<RW>(tile, lane, rowcarry, R);
+  if constexpr (kChan<P>)
+    rows_scan_chan<kBase<P>, RW>(tile, lane, p, sm.bin_of, rowcarry, R);
+  else
+    rows_scan<RW>(tile, lane, rowcarry, R);
   __syncwarp();
   if (lane == 0) mbar_arrive(&sm.empty[s]);  // the tile is consumed: refill the stage
   // a5: running column sums S'(row i) down the warp's rows -> TMEM
@@ -1785,7 +2115,7 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
   bool ended = false;
   for (;;) {
     if (!ended) {
-      if (pass_a<P, CL>(sm, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
+      if (pass_a<P, CL>(sm, p, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
         ++qa;
       else
         ended = true;
@@ -1910,7 +2240,7 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
 
 template <int P, int CL, bool kTMA, bool kVecOut, bool kEx = false>
 __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
-    sat_tile_kernel(const __grid_constant__ CUtensorMap map, const KParams p) {
+    sat_tile_kernel(const __grid_constant__ CUtensorMap map, const __grid_constant__ KParams p) {
   using C = Cfg<P>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   Smem<P, CL>& sm = *reinterpret_cast<Smem<P, CL>*>(smem_raw);
@@ -1918,6 +2248,9 @@ __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
   const int lane = threadIdx.x & 31;
   const uint32_t rank = CL > 1 ? cluster_rank() : 0;
 
+  if constexpr (kBase<P> == P8UHIST4) {
+    for (int i = threadIdx.x; i < 256; i += blockDim.x) sm.bin_of[i] = p.bin_of[i];
+  }
   if (threadIdx.x == 0) {
     for (int s = 0; s < C::NSTAGE; ++s) {
       mbar_init(&sm.full[s], 1);
@@ -1964,7 +2297,7 @@ __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
     typename Agg<kBase<P>>::Acc L = typename Agg<kBase<P>>::Acc(0);
     for (uint32_t q = 0;; ++q) {
       mbar_wait(&sm.full[q % Cfg<P>::NSTAGE], (q / Cfg<P>::NSTAGE) & 1);
-      if (!aggregate_step<P, CL>(sm, rank, q, L, lane)) break;
+      if (!aggregate_step<P, CL>(sm, p, rank, q, L, lane)) break;
     }
   } else if (warp == kOffWarp<P>) {
     for (uint32_t q = 0;; ++q) {

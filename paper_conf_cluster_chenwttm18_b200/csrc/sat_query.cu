@@ -158,6 +158,44 @@ sat_status launch_box(const void* sat, void* out, int64_t h, int64_t w, int64_t 
   return e == cudaSuccess ? SAT_OK : sat::cuda_fail(e, "box_kernel launch");
 }
 
+// Multi-channel SATs (SAT_8U_SQ: K = 2, SAT_8U_HIST4: K = 4): the same
+// four-corner identity per channel, mod 2^32; out is [n][K] uint32.
+template <int K>
+__global__ void rect_sums_chan_kernel(const char* sat, int64_t pitch, int64_t h, int64_t w,
+                                      const int4* rects, int64_t n, uint32_t* out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int4 r = rects[i];
+    const int64_t y0 = std::min<int64_t>(std::max<int64_t>(r.x, 0), h);
+    const int64_t x0 = std::min<int64_t>(std::max<int64_t>(r.y, 0), w);
+    const int64_t y1 = std::min<int64_t>(std::max<int64_t>(r.z, 0), h);
+    const int64_t x1 = std::min<int64_t>(std::max<int64_t>(r.w, 0), w);
+#pragma unroll
+    for (int c = 0; c < K; ++c) {
+      uint32_t v = 0;
+      if (y1 > y0 && x1 > x0) {
+        const uint32_t d = at<int32_t>(sat, pitch, y1 - 1, (x1 - 1) * K + c);
+        const uint32_t b = y0 > 0 ? at<int32_t>(sat, pitch, y0 - 1, (x1 - 1) * K + c) : 0u;
+        const uint32_t cc = x0 > 0 ? at<int32_t>(sat, pitch, y1 - 1, (x0 - 1) * K + c) : 0u;
+        const uint32_t a = (y0 > 0 && x0 > 0) ? at<int32_t>(sat, pitch, y0 - 1, (x0 - 1) * K + c) : 0u;
+        v = (d - b) - (cc - a);
+      }
+      out[i * K + c] = v;
+    }
+  }
+}
+
+template <int K>
+sat_status launch_rects_chan(const void* sat, int64_t sp, int64_t h, int64_t w, const void* rects,
+                             int64_t n, void* out, cudaStream_t s) {
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 16);
+  rect_sums_chan_kernel<K><<<grid, 256, 0, s>>>(static_cast<const char*>(sat), sp, h, w,
+                                                static_cast<const int4*>(rects), n,
+                                                static_cast<uint32_t*>(out));
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? SAT_OK : sat::cuda_fail(e, "rect_sums_chan_kernel launch");
+}
+
 template <typename T>
 sat_status launch_rects(const void* sat, int64_t sp, int64_t h, int64_t w, const void* rects,
                         int64_t n, void* out, cudaStream_t s) {
@@ -200,8 +238,8 @@ sat_status sat_rect_sums(sat_plan plan, const void* sat, int64_t h, int64_t w,
   if (!rects || !out) return sat::fail(SAT_ERR_INVALID_ARGUMENT, "NULL rects or out");
   if ((uintptr_t)rects % 16 != 0)
     return sat::fail(SAT_ERR_INVALID_ARGUMENT, "rects must be 16-byte aligned int32[n][4]");
-  if ((uintptr_t)out % sat::out_size(pair) != 0)
-    return sat::fail(SAT_ERR_INVALID_ARGUMENT, "out misaligned");
+  const size_t ob = sat::multi_channel(pair) ? 4 : sat::out_size(pair);  // channels are u32
+  if ((uintptr_t)out % ob != 0) return sat::fail(SAT_ERR_INVALID_ARGUMENT, "out misaligned");
   sat::DeviceGuard g(plan->device);
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   if (h == 0 || w == 0) {  // every rectangle is empty
@@ -209,6 +247,10 @@ sat_status sat_rect_sums(sat_plan plan, const void* sat, int64_t h, int64_t w,
     return e == cudaSuccess ? SAT_OK : sat::cuda_fail(e, "cudaMemsetAsync");
   }
   switch (pair) {
+    case SAT_8U_SQ:
+      return launch_rects_chan<2>(sat, sat_pitch_bytes, h, w, rects, n, out, s);
+    case SAT_8U_HIST4:
+      return launch_rects_chan<4>(sat, sat_pitch_bytes, h, w, rects, n, out, s);
     case SAT_8U_32S:
     case SAT_32S_32S:
       return launch_rects<int32_t>(sat, sat_pitch_bytes, h, w, rects, n, out, s);
@@ -227,6 +269,8 @@ sat_status sat_box_filter(sat_plan plan, const void* sat, void* out, int64_t h, 
   sat_status st = check_sat_args(plan, sat, h, w, sat_pitch_bytes, pair);
   if (st != SAT_OK) return st;
   if (ry < 0 || rx < 0) return sat::fail(SAT_ERR_INVALID_ARGUMENT, "negative radius");
+  if (sat::multi_channel(pair))
+    return sat::fail(SAT_ERR_UNSUPPORTED, "box filter: single-channel SATs only");
   if (h == 0 || w == 0) return SAT_OK;
   const int64_t sb = (int64_t)sat::out_size(pair);
   if (!out || out_pitch_bytes < w * sb || out_pitch_bytes % sb != 0 || (uintptr_t)out % sb != 0)

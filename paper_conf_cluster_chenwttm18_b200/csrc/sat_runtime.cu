@@ -36,10 +36,13 @@ sat_status cuda_fail(cudaError_t e, const char* what) {
               what, cudaGetErrorName(e), cudaGetErrorString(e));
 }
 
+bool multi_channel(sat_pair p) { return p == SAT_8U_SQ || p == SAT_8U_HIST4; }
 size_t in_size(sat_pair p) {
-  return (p == SAT_8U_32S || p == SAT_8U_32F) ? 1 : (p == SAT_64F_64F ? 8 : 4);
+  return (p == SAT_8U_32S || p == SAT_8U_32F || multi_channel(p)) ? 1 : (p == SAT_64F_64F ? 8 : 4);
 }
-size_t out_size(sat_pair p) { return p == SAT_64F_64F ? 8 : 4; }
+size_t out_size(sat_pair p) {
+  return p == SAT_64F_64F || p == SAT_8U_SQ ? 8 : p == SAT_8U_HIST4 ? 16 : 4;
+}
 int tile_w(sat_pair p) {
   switch (p) {
     case SAT_8U_32S: return Cfg<P8U32S>::TW;
@@ -47,6 +50,8 @@ int tile_w(sat_pair p) {
     case SAT_64F_64F: return Cfg<P64F64F>::TW;
     case SAT_8U_32F: return Cfg<P8U32F>::TW;
     case SAT_32S_32S: return Cfg<P32S32S>::TW;
+    case SAT_8U_SQ: return Cfg<P8USQ>::TW;
+    case SAT_8U_HIST4: return Cfg<P8UHIST4>::TW;
   }
   return 1;
 }
@@ -57,6 +62,8 @@ int tile_h(sat_pair p) {
     case SAT_64F_64F: return Cfg<P64F64F>::TH;
     case SAT_8U_32F: return Cfg<P8U32F>::TH;
     case SAT_32S_32S: return Cfg<P32S32S>::TH;
+    case SAT_8U_SQ: return Cfg<P8USQ>::TH;
+    case SAT_8U_HIST4: return Cfg<P8UHIST4>::TH;
   }
   return 1;
 }
@@ -86,7 +93,7 @@ template <int P>
 static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
                            int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
                            const void* carry_in, cudaStream_t stream, const ExSpec* ex,
-                           const ChainSpec* chain) {
+                           const ChainSpec* chain, const HistSpec* hist) {
   using C = Cfg<P>;
   const bool tma = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
                    pl->force_generic == 0;
@@ -111,13 +118,19 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.chain_ack_out = chain ? chain->ack_out : nullptr;
   kp.chain_ack_in = chain ? chain->ack_in : nullptr;
   kp.chain_epoch = chain ? chain->epoch : 0;
+  memset(kp.bin_of, 0, sizeof(kp.bin_of));
+  kp.bin0 = 0;
+  if (hist) {
+    memcpy(kp.bin_of, hist->bin_of, sizeof(kp.bin_of));
+    kp.bin0 = hist->bin0;
+  }
 
   CUtensorMap map;
   memset(&map, 0, sizeof(map));
   if (tma) {
     EncodeTiledFn enc = get_encode();
     if (!enc) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
-    const CUtensorMapDataType dt = (kBase<P> == P8U32S || kBase<P> == P8U32F)
+    const CUtensorMapDataType dt = (kBase<P> == P8U32S || kBase<P> == P8U32F || kChan<P>)
                                        ? CU_TENSOR_MAP_DATA_TYPE_UINT8
                                    : kBase<P> == P32F32F ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
                                    : kBase<P> == P32S32S ? CU_TENSOR_MAP_DATA_TYPE_UINT32
@@ -203,9 +216,16 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
     smem = sizeof(Smem<P, 4>);
     cfg.dynamicSmemBytes = smem;
     e = cudaLaunchKernelEx(&cfg, sat_tile_kernel<P, 4, true, true, false>, map, kp);
-  } else if (ex) {
-    if (CL == 4) SAT_LAUNCH_CL(4, true) else SAT_LAUNCH_CL(8, true)
-  } else if (CL == 2) SAT_LAUNCH_CL(2, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
+  } else {
+    if constexpr (!kChan<P>) {
+      if (ex) {
+        if (CL == 4) SAT_LAUNCH_CL(4, true) else SAT_LAUNCH_CL(8, true)
+      }
+    }
+    if (!ex) {
+      if (CL == 2) SAT_LAUNCH_CL(2, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
+    }
+  }
 #undef SAT_LAUNCH_CL
   if (e != cudaSuccess) return cuda_fail(e, "sat_tile_kernel launch");
   e = cudaGetLastError();
@@ -291,11 +311,18 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
 static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
                                   int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
                                   const void* carry_in, cudaStream_t stream, const ExSpec* ex,
-                                  const ChainSpec* chain);
+                                  const ChainSpec* chain, const HistSpec* hist);
 
 sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w, int64_t ip,
                   int64_t op, int64_t iis, int64_t ois, int64_t batch, const void* carry_in,
-                  cudaStream_t stream, const ExSpec* ex, const ChainSpec* chain) {
+                  cudaStream_t stream, const ExSpec* ex, const ChainSpec* chain,
+                  const HistSpec* hist) {
+  if (multi_channel(pl->pair) && (carry_in || ex || chain))
+    return fail(SAT_ERR_UNSUPPORTED,
+                "the multi-channel pairs support sat_compute / _batched only (no carry-in, "
+                "exclusive layout or chained bands)");
+  if (pl->pair == SAT_8U_HIST4 && !hist)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "SAT_8U_HIST4 needs bins: use sat_compute_hist4");
   // Tickets and epochs are handed out by the host per launch: a captured
   // launch replayed from a graph would reuse them, so capture is refused.
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
@@ -309,7 +336,8 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
     cudaError_t e = cudaStreamWaitEvent(stream, pl->last_ev, 0);
     if (e != cudaSuccess) return cuda_fail(e, "cudaStreamWaitEvent(plan order)");
   }
-  sat_status st = launch_dispatch(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+  sat_status st =
+      launch_dispatch(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
   if (st == SAT_OK) {
     cudaError_t e = cudaEventRecord(pl->last_ev, stream);
     if (e != cudaSuccess) return cuda_fail(e, "cudaEventRecord(plan order)");
@@ -322,7 +350,7 @@ sat_status launch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t
 static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, int64_t h, int64_t w,
                                   int64_t ip, int64_t op, int64_t iis, int64_t ois, int64_t batch,
                                   const void* carry_in, cudaStream_t stream, const ExSpec* ex,
-                                  const ChainSpec* chain) {
+                                  const ChainSpec* chain, const HistSpec* hist) {
   // Short, wide images: 32-row bands give only H/4 compute warps in total
   // (2 CTAs of 8 warps per SM leave most SMs idle below ~140 bands); 16-row
   // bands (2 rows per warp) double the warps in flight.
@@ -331,33 +359,40 @@ static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, in
   const bool aligned = ((uintptr_t)in % 16 == 0) && (ip % 16 == 0) && (batch == 1 || iis % 16 == 0) &&
                        ((uintptr_t)out % 16 == 0) && (op % 16 == 0) && (batch == 1 || ois % 16 == 0);
   const int sh_env = pl->short_bands;
-  const bool use_short = !ex && aligned && pl->force_generic == 0 && pl->cluster == 0 &&
+  const bool use_short = !ex && !multi_channel(pl->pair) && aligned && pl->force_generic == 0 &&
+                         pl->cluster == 0 &&
                          (sh_env >= 0 ? sh_env == 1 : 2 * bands32 <= (int64_t)pl->num_sms);
   if (use_short) {
     switch (pl->pair) {
       case SAT_8U_32S:
-        return launch_t<P8U32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+        return launch_t<P8U32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
       case SAT_32F_32F:
-        return launch_t<P32F32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+        return launch_t<P32F32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
       case SAT_64F_64F:
-        return launch_t<P64F64F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+        return launch_t<P64F64F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
       case SAT_8U_32F:
-        return launch_t<P8U32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+        return launch_t<P8U32F + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
       case SAT_32S_32S:
-        return launch_t<P32S32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+        return launch_t<P32S32S + kShort>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+      default:
+        break;
     }
   }
   switch (pl->pair) {
     case SAT_8U_32S:
-      return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+      return launch_t<P8U32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
     case SAT_32F_32F:
-      return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+      return launch_t<P32F32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
     case SAT_64F_64F:
-      return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+      return launch_t<P64F64F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
     case SAT_8U_32F:
-      return launch_t<P8U32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+      return launch_t<P8U32F>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
     case SAT_32S_32S:
-      return launch_t<P32S32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain);
+      return launch_t<P32S32S>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+    case SAT_8U_SQ:
+      return launch_t<P8USQ>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+    case SAT_8U_HIST4:
+      return launch_t<P8UHIST4>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
@@ -365,7 +400,8 @@ static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, in
 int cluster_index(int cl) { return cl == 2 ? 0 : cl == 4 ? 1 : 2; }
 
 int default_cluster(int base_pair, int64_t bands) {
-  const bool byte_in = base_pair == P8U32S || base_pair == P8U32F;
+  const bool byte_in = base_pair == P8U32S || base_pair == P8U32F || base_pair == P8USQ ||
+                       base_pair == P8UHIST4;
   return (!byte_in && bands >= 224) ? 8 : 4;
 }
 
@@ -394,7 +430,7 @@ static sat_status configure_cl(sat_plan_st* pl) {
   cudaError_t e0 = cudaFuncSetAttribute(sat_occupancy_proxy<P, CL>,
                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e0 != cudaSuccess) return cuda_fail(e0, "cudaFuncSetAttribute(proxy)");
-  if constexpr (CL == 4 || CL == 8) {
+  if constexpr ((CL == 4 || CL == 8) && !kChan<P>) {
     void (*fx[4])(CUtensorMap, KParams) = {
         sat_tile_kernel<P, CL, false, false, true>, sat_tile_kernel<P, CL, true, false, true>,
         sat_tile_kernel<P, CL, false, true, true>, sat_tile_kernel<P, CL, true, true, true>};
@@ -459,7 +495,8 @@ static sat_status configure_t(sat_plan_st* pl) {
   sat_status st = configure_cl<P, 2>(pl);
   if (st == SAT_OK) st = configure_cl<P, 4>(pl);
   if (st == SAT_OK) st = configure_cl<P, 8>(pl);
-  if (st == SAT_OK) st = configure_short<P>(pl);
+  if constexpr (!kChan<P>)
+    if (st == SAT_OK) st = configure_short<P>(pl);
   return st;
 }
 
@@ -475,6 +512,10 @@ sat_status configure(sat_plan_st* pl) {
       return configure_t<P8U32F>(pl);
     case SAT_32S_32S:
       return configure_t<P32S32S>(pl);
+    case SAT_8U_SQ:
+      return configure_t<P8USQ>(pl);
+    case SAT_8U_HIST4:
+      return configure_t<P8UHIST4>(pl);
   }
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
@@ -572,7 +613,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan out-pointer is NULL");
   *plan = nullptr;
   if (pair != SAT_8U_32S && pair != SAT_32F_32F && pair != SAT_64F_64F && pair != SAT_8U_32F &&
-      pair != SAT_32S_32S)
+      pair != SAT_32S_32S && pair != SAT_8U_SQ && pair != SAT_8U_HIST4)
     return fail(SAT_ERR_INVALID_ARGUMENT, "unknown pair %d", (int)pair);
   if (max_h <= 0 || max_w <= 0 || max_batch <= 0)
     return fail(SAT_ERR_INVALID_ARGUMENT, "plan limits must be positive");
@@ -787,6 +828,26 @@ sat_status sat_compute_exclusive(sat_plan plan, const void* in, void* out, int64
   const ExSpec ex{out_cols, bits};
   return launch(plan, in, out1, hk, w, in_pitch_bytes, out_pitch_bytes, hk * in_pitch_bytes,
                 hk * out_pitch_bytes, 1, nullptr, s, &ex);
+}
+
+sat_status sat_compute_hist4(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
+                             int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                             int64_t in_image_stride_bytes, int64_t out_image_stride_bytes,
+                             int64_t batch, const uint8_t* bin_of, int bin0, void* stream) {
+  if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (plan->pair != SAT_8U_HIST4)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "sat_compute_hist4 needs a SAT_8U_HIST4 plan");
+  if (!bin_of) return fail(SAT_ERR_INVALID_ARGUMENT, "bin table is NULL");
+  bool empty = false;
+  sat_status st = validate(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
+                           in_image_stride_bytes, out_image_stride_bytes, batch, SAT_8U_HIST4, &empty);
+  if (st != SAT_OK || empty) return st;
+  DeviceGuard g(plan->device);
+  const HistSpec hs{bin_of, bin0};
+  return launch(plan, in, out, h, w, in_pitch_bytes, out_pitch_bytes,
+                batch > 1 ? in_image_stride_bytes : h * in_pitch_bytes,
+                batch > 1 ? out_image_stride_bytes : h * out_pitch_bytes, batch, nullptr,
+                static_cast<cudaStream_t>(stream), nullptr, nullptr, &hs);
 }
 
 sat_status sat_compute(sat_plan plan, const void* in, void* out, int64_t h, int64_t w,
