@@ -329,6 +329,19 @@ sat_status sat_dist_colsum(sat_plan plan, const void* in_band, int64_t band_h, i
 sat_status sat_dist_carry(sat_plan plan, const void* gathered, int nranks, int rank, int64_t w,
                           void* carry_out, void* stream);
 
+/* ---------------------------------------------------------------------------
+ * ABLATION, not the product path: the paper's fastest
+ * method, Register-based BRLT-ScanRow run twice (Sec. IV-B;
+ * Alg. 5), ported to sm_100a so the single-pass kernel's
+ * saving can be measured on the same box.  Pass 1 writes the transposed row
+ * prefixes of `in` into `tmp` (w x h, T_B, tmp_pitch_bytes per row of h
+ * elements), pass 2 those of tmp into `out` (h x w): the inclusive SAT, for
+ * SAT_8U_32S / SAT_32F_32F / SAT_64F_64F, at sizeof(T_A) + 3 sizeof(T_B)
+ * bytes per pixel.  Device pointers; stream-ordered. */
+sat_status sat_compute_brlt(sat_pair pair, const void* in, void* out, void* tmp, int64_t h,
+                            int64_t w, int64_t in_pitch_bytes, int64_t out_pitch_bytes,
+                            int64_t tmp_pitch_bytes, void* stream);
+
 /* Static description of a status code. */
 const char* sat_status_string(sat_status s);
 

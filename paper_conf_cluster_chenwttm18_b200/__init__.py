@@ -26,7 +26,7 @@ import threading
 __all__ = ["SatError", "Plan", "sat", "sat_host", "sat_exclusive", "sat_band", "SatComm", "sat_dist",
            "sat_dist_chained", "sat_band_chained", "new_chain_buffer", "chain_bytes", "ChainLink",
            "PeerLink", "SatChain", "rect_sums",
-           "box_filter", "band_partition", "sat_sq", "integral_histogram",
+           "box_filter", "band_partition", "sat_sq", "integral_histogram", "sat_brlt",
            "PAIR_8U_32S", "PAIR_32F_32F", "PAIR_64F_64F", "PAIR_8U_32F", "PAIR_32S_32S", "lib",
            "LIB_PATH"]
 
@@ -73,6 +73,7 @@ def lib():
                     "sat_compute_host": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_exclusive": ([vp, vp, vp, i64, i64, i64, i64, i32, vp, i32, vp], i32),
                     "sat_compute_hist4": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i64, vp, i32, vp], i32),
+                    "sat_compute_brlt": ([i32, vp, vp, vp, i64, i64, i64, i64, i64, vp], i32),
                     "sat_rect_sums": ([vp, vp, i64, i64, i64, vp, i64, vp, i32, vp], i32),
                     "sat_chain_bytes": ([i32, i64], sz),
                     "sat_compute_band_chained": ([vp, vp, vp, i64, i64, i64, i64, vp, vp, vp, ctypes.c_uint32, i32, vp], i32),
@@ -353,6 +354,23 @@ def integral_histogram(x, bins=16, bin_of=None, out=None, plan: Plan | None = No
         _check(lib().sat_compute_hist4(p.handle, x.data_ptr(), o.data_ptr(), H, W, ip,
                                        o.stride(0) * 4, H * ip, H * o.stride(0) * 4, 1, lut, 4 * g,
                                        _stream_ptr(stream, x.device)), "sat_compute_hist4")
+    return out
+
+
+def sat_brlt(x, out=None, tmp=None, stream=None):
+    """ABLATION (not the product path): the paper's two-pass BRLT-ScanRow x 2
+    (PAPER.md Sec. IV-B) for uint8 / float32 / float64 [H, W] CUDA tensors;
+    tmp is the [W, H] intermediate (allocated if None)."""
+    torch = _torch()
+    pair = pair_of_dtype(x.dtype)
+    H, W = x.shape
+    if out is None:
+        out = torch.empty((H, W), dtype=out_dtype(pair), device=x.device)
+    if tmp is None:
+        tmp = torch.empty((W, H), dtype=out_dtype(pair), device=x.device)
+    _check(lib().sat_compute_brlt(pair, x.data_ptr(), out.data_ptr(), tmp.data_ptr(), H, W,
+                                  _row_layout(x)[0], _row_layout(out)[0], _row_layout(tmp)[0],
+                                  _stream_ptr(stream, x.device)), "sat_compute_brlt")
     return out
 
 

@@ -13,6 +13,6 @@ NCCL_INC=$(python -c "import nvidia.nccl,os;print(os.path.join(list(nvidia.nccl.
 cd $TMP/pkg/csrc
 nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -lineinfo -Xcompiler -fPIC -shared \
   --expt-relaxed-constexpr -I $NCCL_INC "${@:3}" -o $ROOT/paper_conf_cluster_chenwttm18_b200/libsat_$NAME.so \
-  sat_runtime.cu sat_host.cu sat_dist.cu sat_query.cu -ldl
+  sat_runtime.cu sat_host.cu sat_dist.cu sat_query.cu $( [ -f sat_brlt.cu ] && echo sat_brlt.cu ) -ldl
 rm -rf $TMP
 echo built libsat_$NAME.so

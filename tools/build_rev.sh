@@ -7,7 +7,7 @@ ROOT=$(cd "$(dirname "$0")/.." && pwd)
 TMP=$(mktemp -d)
 mkdir -p $TMP/include $TMP/pkg/csrc
 SRCS=""
-for f in sat_kernel.cuh sat_runtime.cu sat_host.cu sat_dist.cu sat_query.cu sat_internal.h; do
+for f in sat_kernel.cuh sat_runtime.cu sat_host.cu sat_dist.cu sat_query.cu sat_brlt.cu sat_internal.h; do
   if git -C $ROOT cat-file -e $REV:paper_conf_cluster_chenwttm18_b200/csrc/$f 2>/dev/null; then
     git -C $ROOT show $REV:paper_conf_cluster_chenwttm18_b200/csrc/$f > $TMP/pkg/csrc/$f
     case $f in *.cu) SRCS="$SRCS $f";; esac
