@@ -16,7 +16,7 @@ import subprocess
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-PROFILES = os.path.join(ROOT, "profiles")
+PROFILES = os.environ.get("NCU_SUMMARY_DIR") or os.path.join(ROOT, "profiles")
 KEYS = [
     ("gpu__time_duration.sum", "duration"),
     ("dram__bytes_read.sum", "dram_read"),
@@ -42,9 +42,11 @@ WORKLOAD_OF = {  # prof_one args -> bench workload name
     "p0_1080x1920x1024": "batch-1024x1080x1920-8u32s",
     "p1_65536x65536x1": "huge-65536sq-32f32f",
     "p2_16384x16384x1": "64f-16384sq",
+    "p5_16384x16384x1": "sq-16384sq-8u",
+    "p6_16384x16384x1": "hist4-16384sq-8u",
 }
-IN_B = {0: 1, 1: 4, 2: 8, 3: 1, 4: 4}
-OUT_B = {0: 4, 1: 4, 2: 8, 3: 4, 4: 4}
+IN_B = {0: 1, 1: 4, 2: 8, 3: 1, 4: 4, 5: 1, 6: 1}
+OUT_B = {0: 4, 1: 4, 2: 8, 3: 4, 4: 4, 5: 8, 6: 16}
 
 
 def raw(rep):
