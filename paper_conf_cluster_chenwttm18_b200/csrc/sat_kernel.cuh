@@ -267,6 +267,9 @@ template <int P>
 constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
 // Payload vectors one look-back round lands in shared memory (kLandWords * 8 B
 // per look-back warp).
+#ifndef SAT_LB_LDG
+#define SAT_LB_LDG 0  // look-back reads: 0 bulk copies into shared memory, 1 per-lane loads
+#endif
 #ifndef SAT_LAND_WORDS
 #define SAT_LAND_WORDS 256
 #endif
@@ -374,6 +377,9 @@ __device__ unsigned long long g_sat_tl_v[1024][kTlChunks];    // V_up landed (fi
 __device__ unsigned long long g_sat_tl_ls[1024][kTlChunks];   // leader: gather complete (led chunks)
 __device__ unsigned long long g_sat_tl_lt[1024][kTlChunks];   // leader: prefix known
 __device__ unsigned long long g_sat_tl_ld[1024][kTlChunks];   // leader: V_up sent
+__device__ unsigned int g_sat_tl_rounds[1024][kTlChunks][2];  // leader: look-back rounds, retries
+constexpr int kTlBands = 16384;
+__device__ unsigned long long g_sat_band_t[kTlBands][2];        // every band: first / last pass B
 __device__ __forceinline__ uint64_t tl_now() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -1235,6 +1241,12 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
     for (int e = 0; e < C::E; ++e) V[g][e] = TB(0);
   int64_t j = T - 1;
   uint64_t t_start = 0;
+#if SAT_LB_LDG
+  uint64_t wl[B][C::G][4];
+#define LBW(b, g, e) wl[b][g][e]
+#else
+#define LBW(b, g, e) land[b][((g) * 32 + lane) * 4 + (e)]
+#endif
   for (;;) {
     const int nb = (j - first + 1) < B ? (int)(j - first + 1) : B;
     int kk = nb;  // index of the inclusive vector in this round (nb: none)
@@ -1242,6 +1254,21 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
       __syncwarp();  // every lane is done reading the previous round's landing zone
       SAT_DELAY(31u + (uint32_t)j);
       SAT_PT(i0);
+#if SAT_LB_LDG
+      // every lane loads its own words of the round's vectors straight into
+      // registers (relaxed 16-byte loads: each 8-byte word single-copy atomic)
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+        if (b < nb)
+#pragma unroll
+          for (int g = 0; g < C::G; ++g) {
+            const uint64_t* src = payload_row<P>(p, j - b, chunk) + (g * 32 + lane) * 4;
+            ld_relaxed_v2_u64(src, wl[b][g][0], wl[b][g][1]);
+            ld_relaxed_v2_u64(src + 2, wl[b][g][2], wl[b][g][3]);
+          }
+      SAT_PT(r0);
+      SAT_PT(r1);
+#else
       // lane b fetches vector b (parallel issue); lane 0 arms the barrier.  The
       // previous round's generic reads of the landing zone were consumed before
       // the __syncwarp above, so the async-proxy overwrite cannot overtake them.
@@ -1251,9 +1278,10 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
       SAT_PADD(sm, kPfLbIssue, r0 - i0);
       mbar_wait(land_bar, land_ph);
       SAT_PT(r1);
+      land_ph ^= 1u;
+#endif
       SAT_PADD(sm, kPfLbRoundTime, r1 - r0);
       SAT_PADD(sm, kPfLbRounds, 1);
-      land_ph ^= 1u;
       bool ready = true;
       kk = nb;
       for (int b = 0; b < nb; ++b) {
@@ -1262,7 +1290,7 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
         for (int g = 0; g < C::G; ++g)
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            const uint32_t tg = (uint32_t)(land[b][(g * 32 + lane) * 4 + e] >> 32);
+            const uint32_t tg = (uint32_t)(LBW(b, g, e) >> 32);
             all_incl &= tg == tag_incl;
             all_agg &= tg == tag_agg;
           }
@@ -1275,6 +1303,12 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
           break;
         }
       }
+#ifdef SAT_TIMELINE
+      if (lane == 0 && blockIdx.x < 1024 && chunk < kTlChunks) {
+        g_sat_tl_rounds[blockIdx.x][chunk][0]++;
+        if (!ready) g_sat_tl_rounds[blockIdx.x][chunk][1]++;
+      }
+#endif
       if (ready) break;
       SAT_PADD(sm, kPfLbRetries, 1);
       if (t_start == 0) t_start = gclock();
@@ -1282,7 +1316,10 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
         if (lane == 0) flag_timeout(p);
         return;
       }
-      __nanosleep(32);
+#ifndef SAT_LB_SLEEP
+#define SAT_LB_SLEEP 32
+#endif
+      if (SAT_LB_SLEEP > 0) __nanosleep(SAT_LB_SLEEP);
     }
     const int nsum = kk < nb ? kk + 1 : nb;
     SAT_PADD(sm, kPfLbDepth, nsum);
@@ -1291,7 +1328,7 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
       for (int g = 0; g < C::G; ++g) {
         uint64_t w[4];
 #pragma unroll
-        for (int e = 0; e < 4; ++e) w[e] = land[b][(g * 32 + lane) * 4 + e];
+        for (int e = 0; e < 4; ++e) w[e] = LBW(b, g, e);
         TB t[C::E];
         Tag<kBase<P>>::dec(w, t);
 #pragma unroll
@@ -1300,6 +1337,7 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
     if (kk < nb) break;
     j -= nb;
   }
+#undef LBW
 }
 
 // Chained-band carry vectors: system-scope relaxed 64-bit accesses (peer GPU
@@ -2092,6 +2130,14 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   SAT_PT(t2);
   if (warp == 0) SAT_PADD(sm, kPfComputeFixup, t2 - t1);
 #ifdef SAT_TIMELINE
+  if (warp == 0 && lane == 0 && img >= 0) {
+    const int32_t ch = sm.meta[0][t][3];
+    const int64_t gb = (int64_t)img * p.bands_per_image + sm.meta[0][t][2];
+    if (gb < kTlBands) {
+      if (ch == 0) g_sat_band_t[gb][0] = tl_now();
+      if (ch == p.nchunks - 1) g_sat_band_t[gb][1] = tl_now();
+    }
+  }
   if (warp == 0 && lane == 0 && blockIdx.x < 1024 && img >= 0 && q < kTlChunks &&
       q < (uint32_t)p.nchunks) {
     if (q == 0) g_sat_tl[blockIdx.x][1] = (unsigned long long)sm.meta[0][t][2] +

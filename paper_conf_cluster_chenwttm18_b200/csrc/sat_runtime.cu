@@ -241,6 +241,10 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
     cudaMemcpyFromSymbol(t1, g_sat_tl_ls, sizeof(t1));
     cudaMemcpyFromSymbol(t2, g_sat_tl_lt, sizeof(t2));
     cudaMemcpyFromSymbol(t3, g_sat_tl_ld, sizeof(t3));
+    static unsigned int rr[1024][kTlChunks][2];
+    cudaMemcpyFromSymbol(rr, g_sat_tl_rounds, sizeof(rr));
+    static unsigned int rz[1024][kTlChunks][2];
+    cudaMemcpyToSymbol(g_sat_tl_rounds, rz, sizeof(rz));
     static unsigned long long zero[1024][2 + kTlChunks];
     cudaMemcpyToSymbol(g_sat_tl, zero, sizeof(zero));
     cudaMemcpyToSymbol(g_sat_tl_agg, zero, sizeof(ta));
@@ -250,7 +254,13 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
     cudaMemcpyToSymbol(g_sat_tl_ld, zero, sizeof(ta));
     const char* path = getenv("SAT_TIMELINE_OUT");
     FILE* f = path ? fopen(path, "a") : nullptr;
+    static unsigned long long bt[kTlBands][2];
+    cudaMemcpyFromSymbol(bt, g_sat_band_t, sizeof(bt));
+    static unsigned long long bz[kTlBands][2];
+    cudaMemcpyToSymbol(g_sat_band_t, bz, sizeof(bz));
     if (f) {
+      for (int64_t b = 0; b < kp.total_bands && b < kTlBands; ++b)
+        fprintf(f, "band %lld %llu %llu\n", (long long)b, bt[b][0], bt[b][1]);
       fprintf(f, "launch pair=%d h=%lld w=%lld batch=%lld CL=%d grid=%lld nchunks=%d\n", P,
               (long long)h, (long long)w, (long long)batch, CL, (long long)grid, kp.nchunks);
       const int nc = std::min<int>(kp.nchunks, kTlChunks);
@@ -267,6 +277,8 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
         for (int c = 0; c < nc; ++c) fprintf(f, " %llu", t2[b][c]);
         fprintf(f, "\nld %lld", (long long)b);
         for (int c = 0; c < nc; ++c) fprintf(f, " %llu", t3[b][c]);
+        fprintf(f, "\nrounds %lld", (long long)b);
+        for (int c = 0; c < nc; ++c) fprintf(f, " %u/%u", rr[b][c][0], rr[b][c][1]);
         fprintf(f, "\n");
       }
       fclose(f);
