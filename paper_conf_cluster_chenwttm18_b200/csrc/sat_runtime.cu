@@ -15,6 +15,14 @@
 #include "sat_internal.h"
 #include "sat_kernel.cuh"
 
+// The third cluster size besides 4 and 8: 5, the default for the 8u pairs
+// (clusters of >= 3 CTAs reach 142 of the 148 SMs; 5-CTA clusters place 280
+// CTAs and shorten the look-back chain 1.25x against 4: same-box A/B 16384^2
+// -1.5%, 4096x65536 -4%, 1080p batch -1%; 3 and 6 measured too).
+#ifndef SAT_CLX
+#define SAT_CLX 5
+#endif
+
 namespace {
 
 thread_local char g_last_error[512] = "";
@@ -223,7 +231,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
       }
     }
     if (!ex) {
-      if (CL == 2) SAT_LAUNCH_CL(2, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
+      if (CL == SAT_CLX) SAT_LAUNCH_CL(SAT_CLX, false) else if (CL == 4) SAT_LAUNCH_CL(4, false) else SAT_LAUNCH_CL(8, false)
     }
   }
 #undef SAT_LAUNCH_CL
@@ -409,12 +417,12 @@ static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, in
   return fail(SAT_ERR_INVALID_ARGUMENT, "bad pair");
 }
 
-int cluster_index(int cl) { return cl == 2 ? 0 : cl == 4 ? 1 : 2; }
+int cluster_index(int cl) { return cl == SAT_CLX ? 0 : cl == 4 ? 1 : 2; }
 
 int default_cluster(int base_pair, int64_t bands) {
-  const bool byte_in = base_pair == P8U32S || base_pair == P8U32F || base_pair == P8USQ ||
-                       base_pair == P8UHIST4;
-  return (!byte_in && bands >= 224) ? 8 : 4;
+  if (base_pair == P8U32S || base_pair == P8U32F) return SAT_CLX;
+  if (base_pair == P8USQ || base_pair == P8UHIST4) return 4;
+  return bands >= 224 ? 8 : 4;
 }
 
 int getenv_int(const char* name, int dflt) {
@@ -504,7 +512,7 @@ static sat_status configure_short(sat_plan_st* pl) {
 
 template <int P>
 static sat_status configure_t(sat_plan_st* pl) {
-  sat_status st = configure_cl<P, 2>(pl);
+  sat_status st = configure_cl<P, SAT_CLX>(pl);
   if (st == SAT_OK) st = configure_cl<P, 4>(pl);
   if (st == SAT_OK) st = configure_cl<P, 8>(pl);
   if constexpr (!kChan<P>)
@@ -655,7 +663,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   pl->force_generic = getenv_int("SAT_FORCE_GENERIC", 0);
   {
     const int c = getenv_int("SAT_CLUSTER", 0);
-    pl->cluster = (c == 2 || c == 4 || c == 8) ? c : 0;
+    pl->cluster = (c == SAT_CLX || c == 4 || c == 8) ? c : 0;
   }
   pl->short_bands = getenv_int("SAT_SHORT", -1);
   pl->max_clusters = getenv_int("SAT_MAX_CLUSTERS", 0);
@@ -671,13 +679,17 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   // normal bands) have at most num_sms / 4 tickets.
   int64_t tickets;
   if (pl->cluster > 0) {
-    tickets = (bands + pl->cluster - 1) / pl->cluster;
+    // a forced size other than 4 / 8 still runs exclusive launches with clusters of 4
+    const int64_t c = std::min(pl->cluster, 4);
+    tickets = (bands + c - 1) / c;
+  } else if (pair == SAT_32F_32F || pair == SAT_64F_64F || pair == SAT_32S_32S) {
+    tickets = (std::min<int64_t>(bands, 223) + 3) / 4;  // clusters of 4 below 224 bands
+    tickets = std::max<int64_t>(tickets, (bands + 7) / 8);
   } else {
-    const int base = (int)pair;
-    tickets = (std::min<int64_t>(bands, 223) + 3) / 4;
-    tickets = std::max<int64_t>(tickets, (bands + default_cluster(base, bands) - 1) / default_cluster(base, bands));
-    tickets = std::max<int64_t>(tickets, std::min<int64_t>((2 * bands + 3) / 4, (pl->num_sms + 3) / 4));
+    tickets = (bands + 3) / 4;  // byte pairs: clusters of 5, exclusive launches 4
   }
+  // short-band launches (<= #SMs / 2 normal bands): 16-row bands in clusters of 4
+  tickets = std::max<int64_t>(tickets, std::min<int64_t>((2 * bands + 3) / 4, (pl->num_sms + 3) / 4));
   pl->tickets_cap = tickets;
   const size_t payload_bytes = (size_t)tickets * pl->max_chunks * TW * (out_size(pair) / 4) * 8;
   pl->ws_bytes = 256 + payload_bytes;

@@ -40,7 +40,7 @@ def test_32s_parity(shape):
     assert np.array_equal(y.cpu().numpy(), oracle.sat_32s(x.cpu().numpy()))
 
 
-@pytest.mark.parametrize("env", [{"SAT_CLUSTER": "2"}, {"SAT_CLUSTER": "8"}, {"SAT_SHORT": "1"},
+@pytest.mark.parametrize("env", [{"SAT_CLUSTER": "5"}, {"SAT_CLUSTER": "8"}, {"SAT_SHORT": "1"},
                                  {"SAT_FORCE_GENERIC": "1"}])
 def test_32s_launch_variants(monkeypatch, env):
     torch, sat = _t(), _sat()

@@ -51,7 +51,7 @@ def test_8u32f_parity(shape):
     assert _rel(y.cpu().numpy(), oracle.sat_8u32f(x.cpu().numpy())) <= TOL
 
 
-@pytest.mark.parametrize("env", [{}, {"SAT_CLUSTER": "2"}, {"SAT_CLUSTER": "8"}, {"SAT_SHORT": "1"},
+@pytest.mark.parametrize("env", [{}, {"SAT_CLUSTER": "5"}, {"SAT_CLUSTER": "8"}, {"SAT_SHORT": "1"},
                                  {"SAT_FORCE_GENERIC": "1"}])
 def test_8u32f_launch_variants(monkeypatch, env):
     torch, sat = _t(), _sat()

@@ -63,7 +63,7 @@ def test_sat_sq_wraps_and_batch():
     assert np.array_equal(yb.cpu().numpy(), oracle.sat_sq(xb.cpu().numpy()))
 
 
-@pytest.mark.parametrize("cluster", ["2", "4", "8"])
+@pytest.mark.parametrize("cluster", ["5", "4", "8"])
 def test_sat_sq_cluster_sizes_and_generic_path(monkeypatch, cluster):
     torch, sat = _t(), _sat()
     monkeypatch.setenv("SAT_CLUSTER", cluster)

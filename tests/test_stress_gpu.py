@@ -45,7 +45,7 @@ print("BAD", bad)
 '''
 
 
-@pytest.mark.parametrize("cluster", ["2", "4", "8"])
+@pytest.mark.parametrize("cluster", ["5", "4", "8"])
 def test_lookback_under_injected_delays(cluster):
     if not os.path.exists(DELAY_LIB):
         pytest.skip("libsat_delay.so not built")
