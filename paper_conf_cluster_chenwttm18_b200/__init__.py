@@ -315,6 +315,9 @@ def sat_sq(x, out=None, plan: Plan | None = None, stream=None):
         raise ValueError("sat_sq() takes a uint8 CUDA tensor")
     if out is None:
         out = torch.empty((*x.shape, 2), dtype=torch.int32, device=x.device)
+    if out.dtype != torch.int32 or tuple(out.shape) != (*x.shape, 2) or out.stride(-1) != 1 \
+            or out.stride(-2) != 2:
+        raise ValueError("out must be int32 [..., H, W, 2] with contiguous (S, Q) pairs")
     H, W = x.shape[-2], x.shape[-1]
     N = x.shape[0] if x.dim() == 3 else 1
     if H == 0 or W == 0 or N == 0:

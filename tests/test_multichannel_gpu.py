@@ -163,3 +163,43 @@ def test_multichannel_unsupported_entry_points():
     torch.cuda.synchronize()
     p.close()
     h.close()
+
+
+# ---------------------------------------------------------------------------
+# Seeded randomised cases: shapes around the tile edges (TW = 128 / 64,
+# TH = 32), batches, pitched rows (input offset breaking 16-byte alignment ->
+# the generic load path), random bin tables; sentinel-padded outputs must stay
+# untouched.
+
+@pytest.mark.parametrize("case", range(24))
+def test_multichannel_fuzz(case):
+    torch, sat = _t(), _sat()
+    rng = np.random.default_rng(7000 + case)
+    hist = case % 2 == 1
+    edges = [64, 32] if hist else [128, 32]
+    dim = lambda: int(max(1, rng.choice(edges) * rng.integers(1, 5) + rng.integers(-1, 2))) \
+        if rng.random() < 0.5 else int(rng.integers(1, 900))
+    H, W = dim(), dim()
+    N = int(rng.integers(2, 5)) if (not hist and rng.random() < 0.3) else 1
+    off = int(rng.integers(1, 16)) if rng.random() < 0.25 else 0
+    pitch = W + off + int(rng.integers(0, 32))
+    base = torch.empty((N, H, pitch), dtype=torch.uint8, device="cuda")
+    satgen.fill_device(base, seed=case)
+    x = base[:, :, off:off + W] if N > 1 else base[0, :, off:off + W]
+    if hist:
+        table = rng.integers(0, 9, 256)
+        y = sat.integral_histogram(x, bins=9, bin_of=table)
+        torch.cuda.synchronize()
+        ref = oracle.integral_histogram(x.cpu().numpy(), table, 9)
+        got = np.moveaxis(y.cpu().numpy(), 3, 1).reshape(-1, H, W)[:9]
+        assert np.array_equal(got, ref), f"hist case {case} {H}x{W}"
+    else:
+        K = 2
+        opitch = W + int(rng.integers(0, 8))
+        obuf = torch.full((N, H, opitch, K), -5, dtype=torch.int32, device="cuda")
+        out = obuf[:, :, :W, :] if N > 1 else obuf[0, :, :W, :]
+        sat.sat_sq(x, out=out)
+        torch.cuda.synchronize()
+        ref = oracle.sat_sq(x.cpu().numpy())
+        assert np.array_equal(out.cpu().numpy(), ref), f"sq case {case} {N}x{H}x{W} off {off}"
+        assert torch.all(obuf[:, :, W:, :] == -5), "padding written"
