@@ -13,13 +13,16 @@ pytestmark = pytest.mark.gpu
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 DELAY_LIB = os.path.join(ROOT, "paper_conf_cluster_chenwttm18_b200", "libsat_delay.so")
+# the look-back variant that reads payload words with per-lane ld.relaxed.gpu
+# (8-byte single-copy atomicity guaranteed by PTX) instead of bulk copies
+LDG_LIB = os.path.join(ROOT, "paper_conf_cluster_chenwttm18_b200", "libsat_delay_ldg.so")
 
 SCRIPT = r'''
 import numpy as np, torch, sys
 sys.path.insert(0, sys.argv[1])
 import oracle, satgen
 import paper_conf_cluster_chenwttm18_b200 as sat
-assert sat.LIB_PATH.endswith("libsat_delay.so"), sat.LIB_PATH
+assert "libsat_delay" in sat.LIB_PATH, sat.LIB_PATH
 bad = 0
 for (dt, H, W, N) in [(torch.uint8, 4099, 2311, 1), (torch.float32, 2500, 3000, 1),
                       (torch.float64, 1800, 1700, 1), (torch.uint8, 1080, 900, 5),
@@ -50,6 +53,19 @@ def test_lookback_under_injected_delays(cluster):
     if not os.path.exists(DELAY_LIB):
         pytest.skip("libsat_delay.so not built")
     env = dict(os.environ, SAT_LIBRARY=DELAY_LIB, SAT_CLUSTER=cluster)
+    out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], env=env, capture_output=True,
+                         text=True, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    assert "BAD 0" in out.stdout, out.stdout[-2000:]
+
+
+@pytest.mark.parametrize("cluster", ["5", "4"])
+def test_lookback_ldg_variant_under_injected_delays(cluster):
+    """The same stress on the SAT_LB_LDG=1 build (look-back words read with
+    ld.relaxed.gpu -- the variant whose tag/value atomicity PTX guarantees)."""
+    if not os.path.exists(LDG_LIB):
+        pytest.skip("libsat_delay_ldg.so not built")
+    env = dict(os.environ, SAT_LIBRARY=LDG_LIB, SAT_CLUSTER=cluster)
     out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], env=env, capture_output=True,
                          text=True, timeout=600)
     assert out.returncode == 0, out.stderr[-2000:]
