@@ -33,7 +33,10 @@ struct sat_plan_st {
   size_t ws_bytes = 0;
   unsigned long long* counter = nullptr;  // ticket counter
   uint32_t* err = nullptr;                // device error word (bit 0: a bounded wait timed out)
-  void* payload = nullptr;                // aggregate / inclusive carry vectors
+  void* payload = nullptr;                // aggregate / inclusive carry vectors (integer
+                                          // pairs: the counted reduction tree's nodes)
+  size_t payload_bytes = 0;
+  uint32_t* tree_rd = nullptr;            // tree node read counters [tickets][chunks]
   uint64_t spin_ns = 2000000000ull;       // bounded-wait limit (sat_plan_set_timeout)
   uint32_t epoch = 0;
   uint64_t ticket_base = 0;

@@ -91,7 +91,7 @@ struct Cfg;
 #ifndef SAT_NLW
 #define SAT_NLW 1
 #endif
-constexpr int kNLW = SAT_NLW;                    // leader (look-back) warps
+constexpr int kNLWDefault = SAT_NLW;             // leader (look-back) warps unless Cfg says
 constexpr uint32_t kFull = 0xffffffffu;
 
 // Carry word tag (high 32 bits): (epoch << 2) | st,  st: 1 aggregate, 2 inclusive.
@@ -113,12 +113,23 @@ struct Cfg<P8U32S> {
 #ifndef SAT_NCW8
 #define SAT_NCW8 8
 #endif
-  static constexpr int NCW = SAT_NCW8;   // compute warps, 4 rows each
-  static constexpr int TH = 4 * NCW;     // 32 (2 CTAs per SM) or 64 (1 CTA per SM, 16 warps)
+  static constexpr int NCW = SAT_NCW8;   // compute warps
+#ifndef SAT_TH8
+#define SAT_TH8 32
+#endif
+  static constexpr int TH = SAT_TH8;     // band height (TH / NCW rows per compute warp)
 #ifndef SAT_NST8
 #define SAT_NST8 5
 #endif
   static constexpr int NSTAGE = SAT_NST8;  // TMA prefetch depth (stages free after pass A)
+#ifndef SAT_MINB8
+#define SAT_MINB8 2
+#endif
+  static constexpr int MINB = SAT_MINB8;   // resident CTAs per SM
+#ifndef SAT_NLW8
+#define SAT_NLW8 SAT_NLW
+#endif
+  static constexpr int NLW = SAT_NLW8;     // leader (look-back) warps
 };
 template <>
 struct Cfg<P32F32F> {
@@ -231,6 +242,27 @@ struct Cfg<P8UHIST4> {
 template <int P>
 constexpr bool kChan = kBase<P> == P8USQ || kBase<P> == P8UHIST4;
 
+// Optional per-configuration members: MINB (resident CTAs per SM; default 2,
+// or 1 with more than 8 compute warps) and NLW (leader warps).
+template <int P, class = void>
+struct MinBlocksOf {
+  static constexpr int v = Cfg<P>::NCW > 8 ? 1 : 2;
+};
+template <int P>
+struct MinBlocksOf<P, std::void_t<decltype(Cfg<P>::MINB)>> {
+  static constexpr int v = Cfg<P>::MINB;
+};
+template <int P, class = void>
+struct NlwOf {
+  static constexpr int v = kNLWDefault;
+};
+template <int P>
+struct NlwOf<P, std::void_t<decltype(Cfg<P>::NLW)>> {
+  static constexpr int v = Cfg<P>::NLW;
+};
+template <int P>
+constexpr int kNLW = NlwOf<P>::v;
+
 template <int P>
 struct CfgShort : Cfg<P> {
   static constexpr int TH = Cfg<P>::TH / 2;
@@ -260,7 +292,7 @@ constexpr int kOffWarp = kNCW<P> + 2;
 template <int P>
 constexpr int kFirstLwWarp = kNCW<P> + 3;
 template <int P>
-constexpr int kThreads = (kFirstLwWarp<P> + kNLW) * 32;
+constexpr int kThreads = (kFirstLwWarp<P> + kNLW<P>) * 32;
 
 // Words of one carry payload vector: TW elements * (4 / E) 64-bit words per element.
 template <int P>
@@ -273,8 +305,30 @@ constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
 #ifndef SAT_LAND_WORDS
 #define SAT_LAND_WORDS 256
 #endif
+// Counted reduction tree (integer pairs, SAT_FEN=1): the cross-cluster carry
+// is a Fenwick (binary indexed) tree per image over the clusters' column
+// contributions, built with element-wise atomic bulk reductions (TMA) the
+// moment a cluster's aggregates are gathered; a reader sums the <= log2(D)
+// tree nodes of its prefix in one round -- no chain of inclusive prefixes,
+// so the carry latency does not grow with the depth of the tile column.
+// Each node word is 64 bits: value (bits 0-31, mod 2^32), the carries out of
+// it (bits 32-47) and the number of contributions (bits 48-63), so a word
+// whose count matches the node's writer count holds the complete sum.
+// Exact (wrap-around integer adds commute), hence integer pairs only; the
+// float pairs keep the look-back (fixed summation order).
+#ifndef SAT_FEN
+#define SAT_FEN 0
+#endif
 template <int P>
-constexpr int kLandVecs = (SAT_LAND_WORDS) / kVecWords<P> > 2 ? (SAT_LAND_WORDS) / kVecWords<P> : 2;
+constexpr bool kFen = SAT_FEN != 0 && (kBase<P> == P8U32S || kBase<P> == P32S32S ||
+                                       kBase<P> == P8USQ || kBase<P> == P8UHIST4);
+constexpr uint64_t kFenOne = 1ull << 48;  // one contribution, in a node word's count field
+#ifndef SAT_FEN_LAND
+#define SAT_FEN_LAND 6
+#endif
+template <int P>
+constexpr int kLandVecs = kFen<P> ? (SAT_FEN_LAND)
+                        : (SAT_LAND_WORDS) / kVecWords<P> > 2 ? (SAT_LAND_WORDS) / kVecWords<P> : 2;
 
 // Chunk slots between pass A and pass B (TMEM S', column totals, metadata).
 template <int P>
@@ -291,12 +345,11 @@ constexpr int kNV = Cfg<P>::NSTAGE + kNTot<P>;
 template <int P>
 constexpr int kTmemColsPerWarp =
     (Cfg<P>::TH / kNCW<P>) * Cfg<P>::G * Cfg<P>::E * (int)(sizeof(typename Cfg<P>::TB) / 4);
-// TMEM columns per CTA: 8 compute warps -> 256 (2 CTAs per SM share the SM's
-// 512 columns); 16 compute warps -> 512 (one CTA per SM).
 template <int P>
-constexpr int kTmemCols = 256 * Cfg<P>::NCW / 8;
+constexpr int kMinBlocks = MinBlocksOf<P>::v;  // resident CTAs per SM
+// TMEM columns per CTA: the SM's 512 columns shared by its resident CTAs.
 template <int P>
-constexpr int kMinBlocks = Cfg<P>::NCW > 8 ? 1 : 2;  // resident CTAs per SM
+constexpr int kTmemCols = 512 / kMinBlocks<P>;
 template <int P>
 constexpr int kTmemColsPerSlot = kTmemColsPerWarp<P> * (kNCW<P> / 4);  // NCW/4 warps per subpartition
 static_assert(kTmemColsPerSlot<P8U32S> * kNTot<P8U32S> <= kTmemCols<P8U32S>, "TMEM budget (8u)");
@@ -321,6 +374,8 @@ struct KParams {
   uint64_t ticket_base;                  // counter value at launch
   unsigned long long* counter;           // ticket counter (workspace)
   void* payload;                         // [tickets][nchunks][kVecWords] status-tagged carries
+                                         // (kFen pairs: the counted reduction tree's nodes)
+  uint32_t* tree_rd;                     // kFen: [tickets][nchunks] node read counters
   const void* carry_in;                  // optional S(r0-1, .) row (W elems of TB) for image starts
   // Exclusive layout (kernels instantiated with kEx): S(y, x) is stored at
   // output row y (out already points at row 1 of the exclusive array) and
@@ -414,9 +469,9 @@ enum ProfSlot {
 // The end-of-work sentinels go up to CL * kNLW - 1 chunks further (the next
 // chunk each leader warp would lead), hence the extra CL * kNLW - 1.
 template <int P, int CL>
-constexpr int kNLeadRaw = (Cfg<P>::NSTAGE + kNTot<P> + CL * kNLW - 1 + CL - 1) / CL;
+constexpr int kNLeadRaw = (Cfg<P>::NSTAGE + kNTot<P> + CL * kNLW<P> - 1 + CL - 1) / CL;
 template <int P, int CL>
-constexpr int kNLead = kNLeadRaw<P, CL> > kNLW ? kNLeadRaw<P, CL> : kNLW;
+constexpr int kNLead = kNLeadRaw<P, CL> > kNLW<P> ? kNLeadRaw<P, CL> : kNLW<P>;
 
 template <int P, int CL>
 struct __align__(128) Smem {
@@ -427,7 +482,8 @@ struct __align__(128) Smem {
   alignas(128) typename C::TB vin[kNV<P>][C::TW];            // V_up of this band (from the leader)
   int32_t meta[kNCW<P>][kNTot<P>][4];              // per warp: (band lo, img, k, chunk) of each slot
   uint32_t tmem_base;                           // TMEM address from tcgen05.alloc
-  alignas(128) uint64_t land[kNLW][kLandVecs<P>][kVecWords<P>];  // look-back landing (bulk copies)
+  alignas(128) uint64_t land[kNLW<P>][kLandVecs<P>][kVecWords<P>];  // look-back landing (bulk copies)
+  alignas(128) uint64_t fstage[kNLW<P>][kFen<P> ? kVecWords<P> : 2];  // tree: staged contribution
   uint64_t full[C::NSTAGE];
   uint64_t empty[C::NSTAGE];
   uint64_t tot_full[kNTot<P>];
@@ -436,7 +492,7 @@ struct __align__(128) Smem {
   int64_t lead_band[kNLead<P, CL>];             // leader: its own band of the slot's chunk (-1: end)
   int32_t lead_chunk[kNLead<P, CL>];
   uint64_t vin_full[kNV<P>];                    // tx: V_up landed in vin
-  uint64_t land_full[kNLW];                     // tx: a look-back round landed
+  uint64_t land_full[kNLW<P>];                     // tx: a look-back round landed
   uint64_t tk_full;                             // tx: ticket landed in tk_slot
   uint64_t tk_empty;                            // leader: peers consumed the ticket
   int64_t tk_slot;
@@ -494,6 +550,41 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       "r"(parity), "r"(0x100000u)
       : "memory");
 }
+
+// Long waits (a warp that typically waits microseconds): non-blocking
+// test_wait polls with an exponential __nanosleep back-off.  The hardware
+// try_wait suspend loop wakes on every mbarrier event of the CTA and re-polls,
+// which burnt ~20% of the 8u kernel's issue slots in spin iterations (ncu).
+#ifndef SAT_BO_MAX
+#define SAT_BO_MAX 256
+#endif
+__device__ __forceinline__ bool mbar_test(uint32_t addr, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(addr), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+  const uint32_t addr = smem_u32(bar);
+  if (mbar_test(addr, parity)) return;
+  uint32_t ns = 32;
+  for (;;) {
+    __nanosleep(ns);
+    if (mbar_test(addr, parity)) return;
+    if (ns < (SAT_BO_MAX)) ns <<= 1;
+  }
+}
+#ifndef SAT_BO_CARRY
+#define SAT_BO_CARRY 0
+#endif
+#ifndef SAT_BO_PROD
+#define SAT_BO_PROD 0
+#endif
 
 __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, uint64_t* bar,
                                             int32_t x, int32_t y, int32_t z, uint64_t policy) {
@@ -679,6 +770,11 @@ __device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&v)[16]) {
       : "r"(taddr)
       : "memory");
 }
+// SAT_DEFER_ST=1: pass A does not wait for its TMEM stores; pass B waits
+// (tcgen05.wait::st) just before it loads a slot back.
+#ifndef SAT_DEFER_ST
+#define SAT_DEFER_ST 0
+#endif
 __device__ __forceinline__ void tmem_wait_st() {
   asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }
@@ -1340,6 +1436,206 @@ __device__ __forceinline__ void lookback(SM& sm, uint64_t (&land)[kLandVecs<P>][
 #undef LBW
 }
 
+// ---------------------------------------------------------------------------
+// Counted reduction tree (kFen pairs).  Image n is covered by the cluster
+// tickets T0(n) .. T1(n) (D(n) = T1 - T0 + 1 of them); cluster T0 + u
+// (u <= D - 2) contributes c_u = the column totals of its bands in image n
+// (its tail segment, plus the image's carry-in row where the segment starts
+// the image).  The carry of cluster T0 + t is the exclusive prefix
+// sum_{u < t} c_u = sum of the Fenwick nodes t, t - lowbit(t), ... (> 0);
+// node i (1 <= i <= D - 1) sums c_u for u in [i - lowbit(i), i), so it is complete
+// when its words count lowbit(i) contributions.  Node i of image n, chunk q
+// lives in the payload at vector (T0(n) + i - 1, q); its readers are the
+// clusters t in [i, min(i + lowbit(i), D)), and the last of them (read
+// counter) zeroes it again, so every launch finds the tree zeroed.
+template <int CL>
+__device__ __forceinline__ int64_t img_first_ticket(const KParams& p, int64_t n) {
+  return (n * p.bands_per_image) / CL;
+}
+template <int CL>
+__device__ __forceinline__ int64_t img_tickets(const KParams& p, int64_t n) {
+  return ((n + 1) * p.bands_per_image - 1) / CL - (n * p.bands_per_image) / CL + 1;
+}
+__device__ __forceinline__ int64_t lowbit(int64_t i) { return i & -i; }
+
+__device__ __forceinline__ void bulk_red_add_u64(void* gdst, const void* ssrc, uint32_t bytes) {
+  asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.u64 [%0], [%1], %2;" ::"l"(gdst),
+               "r"(smem_u32(ssrc)), "r"(bytes)
+               : "memory");
+}
+
+// Add cluster t's contribution c (image n with D clusters, chunk q) to the
+// nodes t + 1, then i + lowbit(i), ... (< D): one bulk reduction per node,
+// issued by lane k for the k-th node, from a staged copy in shared memory.
+template <int P, int CL, class SM>
+__device__ __forceinline__ void tree_update(SM& sm, const KParams& p, int lbw, int64_t n, int64_t t,
+                                            int64_t D, int32_t chunk,
+                                            const typename Cfg<P>::TB (&c)[Cfg<P>::G][Cfg<P>::E],
+                                            int lane) {
+  using C = Cfg<P>;
+  constexpr uint32_t kVecBytes = kVecWords<P> * 8;
+  uint64_t* st = sm.fstage[lbw];
+  SAT_DELAY(101u + (uint32_t)t);
+  // the previous update's reductions have read the staged vector
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+  __syncwarp();
+#pragma unroll
+  for (int g = 0; g < C::G; ++g) {
+    const uint4 u = pack16<typename C::TB, C::E>(c[g]);
+    uint64_t* d = st + (g * 32 + lane) * 4;
+    d[0] = kFenOne | u.x;
+    d[1] = kFenOne | u.y;
+    d[2] = kFenOne | u.z;
+    d[3] = kFenOne | u.w;
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
+  __syncwarp();
+  const int64_t base = img_first_ticket<CL>(p, n) - 1;
+  int k = 0;
+  for (int64_t i = t + 1; i <= D - 1; i += lowbit(i), ++k) {
+    if (k == lane) {
+      bulk_red_add_u64(payload_row<P>(p, base + i, chunk), st, kVecBytes);
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    }
+  }
+}
+
+// Read counters of the nodes a query summed: every reader adds one; the last
+// reader zeroes the node and its counter.  The counter adds are issued in
+// tree_query; tree_release (called after the V_up hand-offs) consumes their
+// results, so their round trip is off the critical path.
+struct TreeRel {
+  uint32_t old;    // this lane's counter value before its add (lane < nodes)
+  int64_t node;    // this lane's node (payload vector index), -1: none
+  uint32_t readers;
+};
+
+template <int P>
+__device__ __forceinline__ void tree_release(const KParams& p, int32_t chunk, const TreeRel& r,
+                                             int lane) {
+  using C = Cfg<P>;
+  const bool last = r.node >= 0 && r.old + 1 == r.readers;
+  uint32_t m = __ballot_sync(kFull, last);
+  while (m) {
+    const int k = __ffs(m) - 1;
+    m &= m - 1;
+    const int64_t node = __shfl_sync(kFull, r.node, k);
+    uint64_t* row = payload_row<P>(p, node, chunk);
+#pragma unroll
+    for (int g = 0; g < C::G; ++g) {
+      uint64_t* d = row + (g * 32 + lane) * 4;
+      st_relaxed_v2_u64(d, 0ull, 0ull);
+      st_relaxed_v2_u64(d + 2, 0ull, 0ull);
+    }
+    if (lane == k) p.tree_rd[node * p.nchunks + chunk] = 0u;
+  }
+}
+
+// V = sum of the nodes t, t - lowbit(t), ... of image n's tree (chunk q), each
+// once it is complete.  Rounds land up to kLandVecs nodes (bulk copies);
+// incomplete nodes are re-read.  Returns the last round's read-counter state.
+template <int P, int CL, class SM>
+__device__ __forceinline__ TreeRel tree_query(SM& sm, uint64_t (&land)[kLandVecs<P>][kVecWords<P>],
+                                              uint64_t* land_bar, uint32_t& land_ph,
+                                              const KParams& p, int64_t n, int64_t t, int64_t D,
+                                              int32_t chunk,
+                                              typename Cfg<P>::TB (&V)[Cfg<P>::G][Cfg<P>::E],
+                                              int lane) {
+  using C = Cfg<P>;
+  using TB = typename C::TB;
+  constexpr uint32_t kVecBytes = kVecWords<P> * 8;
+  constexpr int B = kLandVecs<P>;
+  uint32_t acc[C::G][4];
+#pragma unroll
+  for (int g = 0; g < C::G; ++g)
+#pragma unroll
+    for (int e = 0; e < 4; ++e) acc[g][e] = 0u;
+  const int64_t base = img_first_ticket<CL>(p, n) - 1;
+  TreeRel rel{0u, -1, 0u};
+  int64_t i = t;
+  while (i > 0) {
+    // this round's nodes: lane k < nn owns node k of the round
+    int nn = 0;
+    int64_t mine = -1, ii = i;
+    for (; nn < B && ii > 0; ++nn, ii -= lowbit(ii))
+      if (nn == lane) mine = ii;
+    uint32_t pending = (1u << nn) - 1u;
+    uint64_t t_start = 0;
+    while (pending) {
+      __syncwarp();  // every lane is done reading the previous round's landing zone
+      SAT_DELAY(131u + (uint32_t)i);
+#if SAT_LB_LDG
+      // debug variant: per-lane relaxed loads of every pending node, one at a time
+      for (int k = 0; k < nn; ++k) {
+        if (!(pending >> k & 1u)) continue;
+        const int64_t nk = __shfl_sync(kFull, mine, k);
+        const uint64_t* src = payload_row<P>(p, base + nk, chunk);
+        uint64_t w[C::G][4];
+        bool ok = true;
+#pragma unroll
+        for (int g = 0; g < C::G; ++g) {
+          ld_relaxed_v2_u64(src + (g * 32 + lane) * 4, w[g][0], w[g][1]);
+          ld_relaxed_v2_u64(src + (g * 32 + lane) * 4 + 2, w[g][2], w[g][3]);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) ok &= (w[g][e] >> 48) == (uint64_t)lowbit(nk);
+        }
+        if (__all_sync(kFull, ok)) {
+#pragma unroll
+          for (int g = 0; g < C::G; ++g)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[g][e] += (uint32_t)w[g][e];
+          pending &= ~(1u << k);
+        }
+      }
+#else
+      if (lane == 0) mbar_arrive_expect_tx(land_bar, __popc(pending) * kVecBytes);
+      if (mine > 0 && (pending >> lane & 1u))
+        bulk_g2s(&land[lane][0], payload_row<P>(p, base + mine, chunk), kVecBytes, land_bar);
+      mbar_wait(land_bar, land_ph);
+      land_ph ^= 1u;
+      for (int k = 0; k < nn; ++k) {
+        if (!(pending >> k & 1u)) continue;
+        const uint64_t want = (uint64_t)lowbit(__shfl_sync(kFull, mine, k));
+        bool ok = true;
+#pragma unroll
+        for (int g = 0; g < C::G; ++g)
+#pragma unroll
+          for (int e = 0; e < 4; ++e) ok &= (land[k][(g * 32 + lane) * 4 + e] >> 48) == want;
+        if (__all_sync(kFull, ok)) {
+#pragma unroll
+          for (int g = 0; g < C::G; ++g)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[g][e] += (uint32_t)land[k][(g * 32 + lane) * 4 + e];
+          pending &= ~(1u << k);
+        }
+      }
+#endif
+      if (pending) {
+        if (t_start == 0) t_start = gclock();
+        if (gclock() - t_start > p.spin_ns) {  // bounded wait: flag, go on with what is summed
+          if (lane == 0) flag_timeout(p);
+          pending = 0;
+          mine = -1;  // a node left incomplete is not released (the host clears the tree)
+        } else {
+          __nanosleep(32);
+        }
+      }
+    }
+    // the previous round's counters (more than B nodes: long images only)
+    tree_release<P>(p, chunk, rel, lane);
+    rel.node = mine > 0 ? base + mine : -1;
+    rel.readers = mine > 0 ? (uint32_t)min(lowbit(mine), D - mine) : 0u;
+    rel.old = mine > 0 ? atomicAdd(&p.tree_rd[rel.node * p.nchunks + chunk], 1u) : 0u;
+    i = ii;
+  }
+#pragma unroll
+  for (int g = 0; g < C::G; ++g) {
+    uint4 u = make_uint4(acc[g][0], acc[g][1], acc[g][2], acc[g][3]);
+    unpack16<TB, C::E>(u, V[g]);
+  }
+  return rel;
+}
+
 // Chained-band carry vectors: system-scope relaxed 64-bit accesses (peer GPU
 // memory over NVLink keeps aligned 8-byte stores single-copy atomic, so a word
 // with the expected tag also holds its value).
@@ -1498,10 +1794,33 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
   for (int g = 0; g < C::G; ++g)
 #pragma unroll
     for (int e = 0; e < C::E; ++e) contrib[g][e] = tail_self ? carry0[g][e] + tail[g][e] : tail[g][e];
+  TB Vcl[C::G][C::E];
+  TreeRel rel{0u, -1, 0u};
+  if constexpr (kFen<P>) {
+    // Counted reduction tree: contribute to the tail image's tree, then (as a
+    // reader of the head image) sum this cluster's prefix nodes.
+    if (has_succ) {
+      const int64_t g_last = (g0 + CL < p.total_bands ? g0 + CL : p.total_bands) - 1;
+      const int64_t nt = g_last / bpi;
+      tree_update<P, CL>(sm, p, lbw, nt, T - img_first_ticket<CL>(p, nt), img_tickets<CL>(p, nt),
+                         chunk, contrib, lane);
+    }
+#pragma unroll
+    for (int g = 0; g < C::G; ++g)
+#pragma unroll
+      for (int e = 0; e < C::E; ++e) Vcl[g][e] = TB(0);
+    if (!head_self) {
+      SAT_PT(t2);
+      rel = tree_query<P, CL>(sm, sm.land[lbw], &sm.land_full[lbw], land_ph, p, n0,
+                              T - img_first_ticket<CL>(p, n0), img_tickets<CL>(p, n0), chunk, Vcl,
+                              lane);
+      SAT_PT(t3);
+      SAT_PADD(sm, kPfLbLookback, t3 - t2);
+    }
+  } else {
   // aggregate, or -- when the tail segment starts its image -- already inclusive
   if (has_succ)
     publish<P>(p, payload_row<P>(p, T, chunk), tail_self ? kStIncl : kStAgg, contrib, lane);
-  TB Vcl[C::G][C::E];
 #ifdef SAT_DEBUG_NO_LOOKBACK  // timing experiments only: wrong results, no cross-cluster wait
 #pragma unroll
   for (int g = 0; g < C::G; ++g)
@@ -1524,6 +1843,7 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
     }
     SAT_PT(t3);
     SAT_PADD(sm, kPfLbLookback, t3 - t2);
+  }
   }
 #ifdef SAT_TIMELINE
   if (lane == 0 && blockIdx.x < 1024 && qdbg < kTlChunks) g_sat_tl_lt[blockIdx.x][qdbg] = tl_now();
@@ -1568,6 +1888,7 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
     // The image's bottom row S(r1-1, .) = the tail segment's inclusive value.
     if (!has_succ && p.chain_out != nullptr) chain_publish<P>(p, chunk, run, lane);
   }
+  if constexpr (kFen<P>) tree_release<P>(p, chunk, rel, lane);
 }
 
 template <typename TB>
@@ -1620,7 +1941,7 @@ template <int P, int CL>
 __device__ __forceinline__ void leader_warp(Smem<P, CL>& sm, const KParams& p, int lw,
                                             uint32_t rank, int lane) {
   uint32_t land_ph = 0;
-  for (uint32_t j = lw;; j += kNLW) {
+  for (uint32_t j = lw;; j += kNLW<P>) {
     const int ls = j % kNLead<P, CL>;
     SAT_PT(t0);
     mbar_wait_cluster(&sm.lead_full[ls], (j / kNLead<P, CL>) & 1);
@@ -1639,8 +1960,9 @@ __device__ __forceinline__ void leader_warp(Smem<P, CL>& sm, const KParams& p, i
     if (lane == 0 && blockIdx.x < 1024 && q < kTlChunks) g_sat_tl_ld[blockIdx.x][q] = tl_now();
 #endif
   }
-  // the last node stores must have read their staging buffer before the CTA exits
-  if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  // the last node stores / tree reductions must have read their staging buffer
+  // before the CTA exits
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   __syncwarp();
 }
 
@@ -1872,8 +2194,8 @@ __device__ __forceinline__ bool aggregate_step(Smem<P, CL>& sm, const KParams& p
   if (band < 0) {
     if (lane == 0) {
       const uint32_t jn = q <= rank ? 0u : (q - rank + CL - 1) / CL;
-      for (int i = 0; i < kNLW; ++i) {
-        const uint32_t j = jn + (uint32_t)(((i - (int)(jn % kNLW)) % kNLW + kNLW) % kNLW);
+      for (int i = 0; i < kNLW<P>; ++i) {
+        const uint32_t j = jn + (uint32_t)(((i - (int)(jn % kNLW<P>)) % kNLW<P> + kNLW<P>) % kNLW<P>);
         const int ls = j % kNLead<P, CL>;
         sm.lead_band[ls] = -1;
         mbar_arrive(&sm.lead_full[ls]);
@@ -1981,7 +2303,9 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, const KParams& p, uint32
         put_words<TB>(w, (i * C::G + g) * C::E + e, acc[g][e]);
       }
   tmem_st(tmem_addr(sm, t, warp), w);
+#if !SAT_DEFER_ST
   tmem_wait_st();
+#endif
   // a4: this warp's column totals for the block partial-sum scan.
 #pragma unroll
   for (int g = 0; g < C::G; ++g)
@@ -2055,14 +2379,27 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   constexpr int RW = C::TH / kNCW<P>;
   constexpr int NW = kTmemColsPerWarp<P>;
   const int t = q % kNTot<P>;
+  const int32_t img = sm.meta[warp][t][1];  // written by this warp's pass A
+  uint32_t w[NW];
+#if SAT_DEFER_ST
+  // S' back from TMEM first: the load's latency overlaps the carry wait
+  if (img >= 0) {
+    tmem_wait_st();  // pass A's stores (the latest one an iteration ago) have landed
+    tmem_ld(tmem_addr(sm, t, warp), w);
+  }
+#endif
   SAT_PT(t0);
+#if SAT_BO_CARRY
+  mbar_wait_sleep(&sm.carry_full[t], (q / kNTot<P>) & 1);
+#else
   mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
+#endif
   SAT_PT(t1);
   if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
-  const int32_t img = sm.meta[warp][t][1];
   if (img >= 0) {
-    uint32_t w[NW];
+#if !SAT_DEFER_ST
     tmem_ld(tmem_addr(sm, t, warp), w);
+#endif
     TB off[C::G][C::E];  // V_up + the warps above + nVal (offset warp)
 #pragma unroll
     for (int g = 0; g < C::G; ++g)
@@ -2159,6 +2496,26 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
   for (int i = 0; i < RW; ++i) rowcarry[i] = TB(0);
   uint32_t qa = 0, qb = 0;
   bool ended = false;
+  // Pass B of chunk q runs right after pass A of chunk q + LOOK, at the top of
+  // the next iteration (so pass A's TMEM stores have an iteration to land
+  // before a TMEM load waits for them); before pass A(qa), qa - qb <= LOOK,
+  // i.e. the slot qa reuses (qa - LOOK - 1) has been drained.
+#if SAT_DEFER_ST
+  for (;;) {
+    if (qb < qa && (ended || qa - qb > (uint32_t)C::LOOK)) {
+      pass_b<P, CL, kVecOut, kEx>(sm, p, qb, warp, lane, prevlast);
+      ++qb;
+    }
+    if (!ended) {
+      if (pass_a<P, CL>(sm, p, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
+        ++qa;
+      else
+        ended = true;
+    } else if (qb == qa) {
+      break;
+    }
+  }
+#else
   for (;;) {
     if (!ended) {
       if (pass_a<P, CL>(sm, p, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
@@ -2173,6 +2530,7 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
       break;
     }
   }
+#endif
   // End-of-work sentinel for the offset warp (the slot is free: all pass B done).
   {
     const int t = qa % kNTot<P>;
@@ -2191,7 +2549,10 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
   using C = Cfg<P>;
   using TA = typename C::TA;
   constexpr uint32_t kTileBytes = C::TH * C::TW * sizeof(TA);
-  constexpr uint32_t kTicketLead = 2;  // chunks of the current band still ahead of pass A
+#ifndef SAT_TICKET_LEAD
+#define SAT_TICKET_LEAD 2
+#endif
+  constexpr uint32_t kTicketLead = SAT_TICKET_LEAD;  // chunks of the current band still ahead of pass A
   uint32_t q = 0, draws = 0;
   uint64_t pol = 0;
   if (kTMA) pol = policy_evict_first();
@@ -2232,7 +2593,11 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
     const int32_t nch = done ? 1 : p.nchunks;
     for (int32_t c = 0; c < nch; ++c, ++q) {
       const int s = q % C::NSTAGE;
+#if SAT_BO_PROD
+      mbar_wait_sleep(&sm.empty[s], ((q / C::NSTAGE) & 1) ^ 1u);
+#else
       mbar_wait(&sm.empty[s], ((q / C::NSTAGE) & 1) ^ 1u);
+#endif
       if (done) {
         if (lane == 0) {
           sm.stage_band[s] = -1;
@@ -2308,7 +2673,7 @@ __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
     }
     for (int v = 0; v < kNV<P>; ++v) mbar_init(&sm.vin_full[v], 1);
     for (int i = 0; i < kNLead<P, CL>; ++i) mbar_init(&sm.lead_full[i], 1);
-    for (int i = 0; i < kNLW; ++i) mbar_init(&sm.land_full[i], 1);
+    for (int i = 0; i < kNLW<P>; ++i) mbar_init(&sm.land_full[i], 1);
     mbar_init(&sm.tk_full, 1);
     mbar_init(&sm.tk_empty, CL > 1 ? CL - 1 : 1);
     sm.passA_done = 0;

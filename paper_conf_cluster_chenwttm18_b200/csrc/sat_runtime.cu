@@ -164,7 +164,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   // Look-back workspace: one tagged carry vector per (cluster ticket, chunk).
   {
     const size_t need = (size_t)kp.total_tickets * kp.nchunks * kVecWords<P> * 8;
-    const size_t have = pl->ws_bytes - ((char*)pl->payload - (char*)pl->ws);
+    const size_t have = pl->payload_bytes;
     if (need > have)
       return fail(SAT_ERR_INVALID_ARGUMENT,
                   "problem needs %zu bytes of carry workspace (cluster %d), plan holds %zu", need, CL,
@@ -184,6 +184,12 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.epoch = ++pl->epoch;
   kp.counter = pl->counter;
   kp.payload = pl->payload;
+  kp.tree_rd = pl->tree_rd;
+  if (kFen<P> && (size_t)kp.total_tickets * kp.nchunks > (size_t)pl->tickets_cap * pl->max_chunks)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "problem exceeds the plan's carry-tree counters");
+  if (kFen<P> && kp.bands_per_image / CL + 2 >= (1 << 16))
+    return fail(SAT_ERR_UNSUPPORTED, "image too tall: %lld bands exceed the carry tree's count field",
+                (long long)kp.bands_per_image);
   kp.ticket_base = pl->ticket_base;
 
   const int mode = (tma ? 1 : 0) | (vec ? 2 : 0);
@@ -692,7 +698,10 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   tickets = std::max<int64_t>(tickets, std::min<int64_t>((2 * bands + 3) / 4, (pl->num_sms + 3) / 4));
   pl->tickets_cap = tickets;
   const size_t payload_bytes = (size_t)tickets * pl->max_chunks * TW * (out_size(pair) / 4) * 8;
-  pl->ws_bytes = 256 + payload_bytes;
+  // integer pairs: one read counter per tree node (= per payload vector)
+  const size_t rd_bytes = (size_t)tickets * pl->max_chunks * 4;
+  pl->payload_bytes = payload_bytes;
+  pl->ws_bytes = 256 + payload_bytes + rd_bytes;
   sat_status st = configure(pl);
   if (st == SAT_OK) {
     e = cudaEventCreateWithFlags(&pl->last_ev, cudaEventDisableTiming);
@@ -716,6 +725,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   pl->counter = reinterpret_cast<unsigned long long*>(pl->ws);
   pl->err = reinterpret_cast<uint32_t*>(static_cast<char*>(pl->ws) + 64);
   pl->payload = static_cast<char*>(pl->ws) + 256;
+  pl->tree_rd = reinterpret_cast<uint32_t*>(static_cast<char*>(pl->ws) + 256 + payload_bytes);
   cudaSetDevice(prev);
   *plan = pl;
   return SAT_OK;
@@ -735,6 +745,9 @@ sat_status sat_plan_status(sat_plan plan, void* stream) {
   cudaError_t e = cudaMemcpyAsync(&h, plan->err, 4, cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e == cudaSuccess && h != 0) e = cudaMemsetAsync(plan->err, 0, 4, s);
+  // a timed-out launch may leave carry-tree nodes partly summed: clear the tree
+  if (e == cudaSuccess && h != 0)
+    e = cudaMemsetAsync(plan->payload, 0, plan->ws_bytes - ((char*)plan->payload - (char*)plan->ws), s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return cuda_fail(e, "sat_plan_status");
   if (h & 1u)
