@@ -35,7 +35,8 @@
  *    other than the plan's previous one first waits (cudaStreamWaitEvent) for
  *    that launch, so two streams sharing a plan serialise instead of racing on
  *    the workspace.  Workspace is never re-zeroed per call: carry words carry a
- *    per-call epoch.  Stream capture (CUDA graphs) of a compute call returns
+ *    per-call epoch, and the carry tree's nodes are zeroed again by their last
+ *    reader (after a timed-out launch sat_plan_status clears them).  Stream capture (CUDA graphs) of a compute call returns
  *    SAT_ERR_UNSUPPORTED (tickets and epochs are handed out per launch by the
  *    host).
  *  - Cross-CTA and cross-GPU carry waits are bounded (sat_plan_set_timeout,
@@ -112,6 +113,24 @@ sat_status sat_plan_workspace_bytes(sat_plan plan, size_t* bytes);
 /* Bound (ns, > 0) on every cross-CTA / cross-GPU carry wait of later launches
  * of `plan` (default 2e9).  Errors: INVALID_ARGUMENT (NULL plan, ns == 0). */
 sat_status sat_plan_set_timeout(sat_plan plan, uint64_t ns);
+
+/* Cross-cluster vertical carry of the integer pairs (8u->32s, 32s->32s,
+ * 8u->(S,S^2), integral histogram) -- V_up(x) = S(r0-1, x) of a cluster's
+ * first band, PAPER.md:258-260 (Sec. IV-C, the carries between blocks).
+ *  SAT_CARRY_LOOKBACK  decoupled look-back over epoch-tagged aggregate /
+ *                      inclusive vectors (the float pairs always use it);
+ *  SAT_CARRY_TREE      counted reduction tree: each cluster adds its column
+ *                      totals into the Fenwick nodes above it with TMA bulk
+ *                      reductions, a reader sums <= log2(D) complete nodes
+ *                      (exact: wrap-around integer adds commute);
+ *  SAT_CARRY_AUTO      per launch by shape (default; the tree for images of
+ *                      <= 64 bands and launches of <= one wave of bands).
+ * The initial mode comes from the environment variable SAT_TREE (-1/0/1) read
+ * at plan creation.  Applies to later launches of `plan`.
+ * Errors: INVALID_ARGUMENT (NULL plan, unknown mode), UNSUPPORTED (TREE on a
+ * float pair). */
+typedef enum { SAT_CARRY_AUTO = 0, SAT_CARRY_LOOKBACK = 1, SAT_CARRY_TREE = 2 } sat_carry;
+sat_status sat_plan_set_carry(sat_plan plan, sat_carry mode);
 
 /* Synchronises `stream` and reports (then clears) the plan's device error
  * word: SAT_ERR_TIMEOUT if a bounded carry wait of an earlier launch ran out

@@ -67,6 +67,7 @@ def lib():
                     "sat_plan_destroy": ([vp], i32),
                     "sat_plan_set_timeout": ([vp, ctypes.c_uint64], i32),
                     "sat_plan_status": ([vp, vp], i32),
+                    "sat_plan_set_carry": ([vp, i32], i32),
                     "sat_compute": ([vp, vp, vp, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_batched": ([vp, vp, vp, i64, i64, i64, i64, i64, i64, i64, i32, vp], i32),
                     "sat_compute_band": ([vp, vp, vp, i64, i64, i64, i64, vp, i32, vp], i32),
@@ -168,6 +169,12 @@ class Plan:
     def set_timeout(self, ns: int):
         """Bound every cross-CTA / cross-GPU carry wait of later launches (ns)."""
         _check(lib().sat_plan_set_timeout(self._h, int(ns)), "sat_plan_set_timeout")
+
+    def set_carry(self, mode: str):
+        """Cross-cluster carry of later launches: "auto" (by shape), "lookback"
+        or "tree" (integer pairs; see sat_plan_set_carry)."""
+        m = {"auto": 0, "lookback": 1, "tree": 2}[mode]
+        _check(lib().sat_plan_set_carry(self._h, m), "sat_plan_set_carry")
 
     def status(self, stream=None):
         """Synchronise `stream`; raise SatError(SAT_ERR_TIMEOUT) if a bounded

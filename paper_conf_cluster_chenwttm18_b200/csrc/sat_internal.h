@@ -26,6 +26,7 @@ struct sat_plan_st {
   int short_bands = -1;   // -1 by shape, 0 / 1 forced
   int max_clusters = 0, force_clusters = 0;
   int log = 0;
+  int tree_mode = -1;     // SAT_TREE: integer-pair carries -1 by shape, 0 look-back, 1 tree
   int64_t max_tiles = 0;       // max_batch * bands * chunks of the plan limits (normal bands)
   int64_t tickets_cap = 0;     // cluster tickets the look-back payload holds at the plan's max width
   int64_t max_chunks = 0;
@@ -37,6 +38,7 @@ struct sat_plan_st {
                                           // pairs: the counted reduction tree's nodes)
   size_t payload_bytes = 0;
   uint32_t* tree_rd = nullptr;            // tree node read counters [tickets][chunks]
+  bool lookback_dirty = false;            // a look-back launch left tagged words in the payload
   uint64_t spin_ns = 2000000000ull;       // bounded-wait limit (sat_plan_set_timeout)
   uint32_t epoch = 0;
   uint64_t ticket_base = 0;

@@ -316,8 +316,10 @@ constexpr int kVecWords = Cfg<P>::TW * 4 / Cfg<P>::E;
 // whose count matches the node's writer count holds the complete sum.
 // Exact (wrap-around integer adds commute), hence integer pairs only; the
 // float pairs keep the look-back (fixed summation order).
+// SAT_FEN: 1 compiles the tree into the integer-pair kernels next to the
+// look-back; KParams::tree selects it per launch (the runtime's shape rule).
 #ifndef SAT_FEN
-#define SAT_FEN 0
+#define SAT_FEN 1
 #endif
 template <int P>
 constexpr bool kFen = SAT_FEN != 0 && (kBase<P> == P8U32S || kBase<P> == P32S32S ||
@@ -376,6 +378,9 @@ struct KParams {
   void* payload;                         // [tickets][nchunks][kVecWords] status-tagged carries
                                          // (kFen pairs: the counted reduction tree's nodes)
   uint32_t* tree_rd;                     // kFen: [tickets][nchunks] node read counters
+  int32_t tree;                          // kFen pairs: 1 carries by the tree, 0 by the look-back
+  uint32_t ticket_lead;                  // draw the next ticket when pass A is this many
+                                         // chunks from the end of the issued tiles
   const void* carry_in;                  // optional S(r0-1, .) row (W elems of TB) for image starts
   // Exclusive layout (kernels instantiated with kEx): S(y, x) is stored at
   // output row y (out already points at row 1 of the exclusive array) and
@@ -818,6 +823,25 @@ __device__ __forceinline__ TB get_words(const uint32_t (&w)[N], int idx) {
   }
 }
 
+// One Kogge-Stone step in place, v += v(lane - d) for lane >= d (Alg. 3,
+// reading R10): shfl.up's in-range predicate guards the add -- two
+// instructions per step (the C++ form compiled to shuffle + predicated add +
+// move).  Same operation and order, so results are unchanged.
+__device__ __forceinline__ void ks_step(uint32_t& v, int d) {
+  asm("{\n\t.reg .pred p;\n\t.reg .b32 t;\n\t"
+      "shfl.sync.up.b32 t|p, %0, %1, 0, -1;\n\t"
+      "@p add.u32 %0, %0, t;\n\t}"
+      : "+r"(v)
+      : "r"(d));
+}
+__device__ __forceinline__ void ks_step(float& v, int d) {
+  asm("{\n\t.reg .pred p;\n\t.reg .f32 t;\n\t"
+      "shfl.sync.up.b32 t|p, %0, %1, 0, -1;\n\t"
+      "@p add.rn.f32 %0, %0, t;\n\t}"
+      : "+f"(v)
+      : "r"(d));
+}
+
 // ---------------------------------------------------------------------------
 // a2 + a3: scan the RW rows a warp owns, all rows advancing through the
 // Kogge-Stone stages together (RW-way ILP on the shuffle latency).  Produces
@@ -843,14 +867,9 @@ __device__ __forceinline__ void rows_scan(const uint8_t* tile, int lane, uint32_
     inc[i] = own[i];
   }
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {  // a3: Alg. 3, lane >= d (reading R10)
-    uint32_t o[RW];
+  for (int d = 1; d < 32; d <<= 1)  // a3: Alg. 3, lane >= d (reading R10)
 #pragma unroll
-    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
-#pragma unroll
-    for (int i = 0; i < RW; ++i)
-      if (lane >= d) inc[i] += o[i];
-  }
+    for (int i = 0; i < RW; ++i) ks_step(inc[i], d);
 #pragma unroll
   for (int i = 0; i < RW; ++i) {
     const uint32_t tot = __shfl_sync(kFull, inc[i], 31);
@@ -886,14 +905,9 @@ __device__ __forceinline__ void rows_scan(const float* tile, int lane, float (&r
     inc[i] = p[i][3];
   }
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {  // Alg. 3
-    float o[RW];
+  for (int d = 1; d < 32; d <<= 1)  // Alg. 3
 #pragma unroll
-    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
-#pragma unroll
-    for (int i = 0; i < RW; ++i)
-      if (lane >= d) inc[i] += o[i];
-  }
+    for (int i = 0; i < RW; ++i) ks_step(inc[i], d);
 #pragma unroll
   for (int i = 0; i < RW; ++i) {
     const float tot = __shfl_sync(kFull, inc[i], 31);
@@ -972,14 +986,9 @@ __device__ __forceinline__ void rows_scan(const uint32_t* tile, int lane, uint32
     inc[i] = p[i][3];
   }
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {  // Alg. 3
-    uint32_t o[RW];
+  for (int d = 1; d < 32; d <<= 1)  // a3: Alg. 3, lane >= d (reading R10)
 #pragma unroll
-    for (int i = 0; i < RW; ++i) o[i] = __shfl_up_sync(kFull, inc[i], d);
-#pragma unroll
-    for (int i = 0; i < RW; ++i)
-      if (lane >= d) inc[i] += o[i];
-  }
+    for (int i = 0; i < RW; ++i) ks_step(inc[i], d);
 #pragma unroll
   for (int i = 0; i < RW; ++i) {
     const uint32_t tot = __shfl_sync(kFull, inc[i], 31);
@@ -1796,7 +1805,7 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
     for (int e = 0; e < C::E; ++e) contrib[g][e] = tail_self ? carry0[g][e] + tail[g][e] : tail[g][e];
   TB Vcl[C::G][C::E];
   TreeRel rel{0u, -1, 0u};
-  if constexpr (kFen<P>) {
+  if (kFen<P> && p.tree) {
     // Counted reduction tree: contribute to the tail image's tree, then (as a
     // reader of the head image) sum this cluster's prefix nodes.
     if (has_succ) {
@@ -1888,7 +1897,7 @@ __device__ __forceinline__ void leader_chunk(Smem<P, CL>& sm, const KParams& p, 
     // The image's bottom row S(r1-1, .) = the tail segment's inclusive value.
     if (!has_succ && p.chain_out != nullptr) chain_publish<P>(p, chunk, run, lane);
   }
-  if constexpr (kFen<P>) tree_release<P>(p, chunk, rel, lane);
+  if (kFen<P> && p.tree) tree_release<P>(p, chunk, rel, lane);
 }
 
 template <typename TB>
@@ -1997,12 +2006,16 @@ template <typename T>
 __device__ __forceinline__ T warp_incl(T v, int lane) {
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
-    T o;
-    if constexpr (IsChan<T>::value)
-      o = shfl_up(v, d);
-    else
-      o = __shfl_up_sync(kFull, v, d);
-    if (lane >= d) v += o;
+    if constexpr (std::is_same<T, uint32_t>::value || std::is_same<T, float>::value) {
+      ks_step(v, d);
+    } else {
+      T o;
+      if constexpr (IsChan<T>::value)
+        o = shfl_up(v, d);
+      else
+        o = __shfl_up_sync(kFull, v, d);
+      if (lane >= d) v += o;
+    }
   }
   return v;
 }
@@ -2549,10 +2562,7 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
   using C = Cfg<P>;
   using TA = typename C::TA;
   constexpr uint32_t kTileBytes = C::TH * C::TW * sizeof(TA);
-#ifndef SAT_TICKET_LEAD
-#define SAT_TICKET_LEAD 2
-#endif
-  constexpr uint32_t kTicketLead = SAT_TICKET_LEAD;  // chunks of the current band still ahead of pass A
+  const uint32_t kTicketLead = p.ticket_lead;  // chunks of the current band still ahead of pass A
   uint32_t q = 0, draws = 0;
   uint64_t pol = 0;
   if (kTMA) pol = policy_evict_first();

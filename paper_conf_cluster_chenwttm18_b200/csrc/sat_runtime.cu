@@ -185,11 +185,40 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   kp.counter = pl->counter;
   kp.payload = pl->payload;
   kp.tree_rd = pl->tree_rd;
-  if (kFen<P> && (size_t)kp.total_tickets * kp.nchunks > (size_t)pl->tickets_cap * pl->max_chunks)
-    return fail(SAT_ERR_INVALID_ARGUMENT, "problem exceeds the plan's carry-tree counters");
-  if (kFen<P> && kp.bands_per_image / CL + 2 >= (1 << 16))
-    return fail(SAT_ERR_UNSUPPORTED, "image too tall: %lld bands exceed the carry tree's count field",
-                (long long)kp.bands_per_image);
+  kp.tree = 0;
+  // Ticket pacing: a CTA draws its next band when pass A is kp.ticket_lead
+  // chunks from the end of what it has issued.  Short bands (batches of small
+  // frames) draw early, so the next band's tiles and carries are under way
+  // while the current one drains (1080p batch -7..9%); long bands draw late
+  // (a drawn band must not queue behind a whole band).
+#ifndef SAT_TICKET_LEAD
+#define SAT_TICKET_LEAD 0
+#endif
+  kp.ticket_lead = SAT_TICKET_LEAD > 0 ? SAT_TICKET_LEAD
+                                       : (kp.nchunks <= 16 ? (uint32_t)C::NSTAGE : 2u);
+  if constexpr (kFen<P>) {
+    // Carry mechanism (integer pairs): the counted reduction tree where the
+    // look-back chain is what paces the launch -- images of few bands
+    // (batches: every band start waits for its carry) and launches of at
+    // most one wave of bands; the look-back where bands run two waves and
+    // more (measured).  SAT_TREE=0/1 forces it.
+    const int64_t slots = (int64_t)pl->active_clusters[kBase<P>][cluster_index(CL)][3] * CL;
+    const bool tree_shape = kp.bands_per_image <= 64 || kp.total_bands <= slots;
+    kp.tree = pl->tree_mode >= 0 ? pl->tree_mode : (tree_shape ? 1 : 0);
+    if (kp.tree && (size_t)kp.total_tickets * kp.nchunks > (size_t)pl->tickets_cap * pl->max_chunks)
+      return fail(SAT_ERR_INVALID_ARGUMENT, "problem exceeds the plan's carry-tree counters");
+    if (kp.tree && kp.bands_per_image / CL + 2 >= (1 << 16)) kp.tree = 0;  // count field: look-back
+    // The tree needs zeroed nodes (every tree launch leaves them zeroed); the
+    // look-back leaves tagged words in the same workspace: clear the part a
+    // tree launch uses when the plan's previous carry launch looked back.
+    if (kp.tree && pl->lookback_dirty) {
+      const size_t vecs = (size_t)kp.total_tickets * kp.nchunks;
+      cudaError_t e = cudaMemsetAsync(pl->payload, 0, vecs * kVecWords<P> * 8, stream);
+      if (e == cudaSuccess) e = cudaMemsetAsync(pl->tree_rd, 0, vecs * 4, stream);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(carry tree)");
+    }
+    pl->lookback_dirty = !kp.tree;
+  }
   kp.ticket_base = pl->ticket_base;
 
   const int mode = (tma ? 1 : 0) | (vec ? 2 : 0);
@@ -328,9 +357,9 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   if (pl->log)
     fprintf(stderr,
             "[libsat] pair=%d %lldx%lld batch=%lld tma=%d vec=%d cluster=%d grid=%lld smem=%zu "
-            "epoch=%u\n",
+            "epoch=%u tree=%d\n",
             P, (long long)h, (long long)w, (long long)batch, (int)tma, (int)vec, CL, (long long)grid,
-            smem, kp.epoch);
+            smem, kp.epoch, (int)kp.tree);
   return SAT_OK;
 }
 
@@ -675,6 +704,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
   pl->max_clusters = getenv_int("SAT_MAX_CLUSTERS", 0);
   pl->force_clusters = getenv_int("SAT_FORCE_CLUSTERS", 0);
   pl->log = getenv_int("SAT_LOG", 0);
+  pl->tree_mode = getenv_int("SAT_TREE", -1);
   const int64_t TH = tile_h(pair), TW = tile_w(pair);
   const int64_t bands = max_batch * ((max_h + TH - 1) / TH);
   pl->max_chunks = (max_w + TW - 1) / TW;
@@ -734,6 +764,18 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
 sat_status sat_plan_set_timeout(sat_plan plan, uint64_t ns) {
   if (!plan || ns == 0) return fail(SAT_ERR_INVALID_ARGUMENT, "NULL plan or zero timeout");
   plan->spin_ns = ns;
+  return SAT_OK;
+}
+
+sat_status sat_plan_set_carry(sat_plan plan, sat_carry mode) {
+  if (!plan) return fail(SAT_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (mode != SAT_CARRY_AUTO && mode != SAT_CARRY_LOOKBACK && mode != SAT_CARRY_TREE)
+    return fail(SAT_ERR_INVALID_ARGUMENT, "unknown carry mode %d", (int)mode);
+  const bool integer = plan->pair == SAT_8U_32S || plan->pair == SAT_32S_32S ||
+                       plan->pair == SAT_8U_SQ || plan->pair == SAT_8U_HIST4;
+  if (mode == SAT_CARRY_TREE && !integer)
+    return fail(SAT_ERR_UNSUPPORTED, "the carry tree is for the integer pairs only");
+  plan->tree_mode = mode == SAT_CARRY_AUTO ? -1 : mode == SAT_CARRY_TREE ? 1 : 0;
   return SAT_OK;
 }
 

@@ -1,8 +1,11 @@
-"""Carry-tree stress: the -DSAT_DEBUG_DELAY build sleeps a pseudo-random 0..4 us
-before every node publication, tree round and DSMEM hand-off, so late
-predecessors, half-written nodes and retries all occur (tall images reach
-tree level 3; 40 two-band frames put several whole images in one cluster).  Run
-in a subprocess (the library is chosen at import through SAT_LIBRARY)."""
+"""Carry stress: the -DSAT_DEBUG_DELAY build sleeps a pseudo-random 0..4 us
+before every carry publication, look-back round, tree update / query round and
+DSMEM hand-off, so late predecessors, half-summed tree nodes, mixed
+aggregate/inclusive windows and retries all occur (40 two-band frames put
+several whole images in one cluster).  Both cross-cluster carry mechanisms run:
+the decoupled look-back (SAT_TREE=0) and, for the integer pairs, the counted
+reduction tree (SAT_TREE=1).  Run in a subprocess (the library is chosen at
+import through SAT_LIBRARY)."""
 import os
 import subprocess
 import sys
@@ -48,24 +51,26 @@ print("BAD", bad)
 '''
 
 
-@pytest.mark.parametrize("cluster", ["5", "4", "8"])
-def test_lookback_under_injected_delays(cluster):
+@pytest.mark.parametrize("cluster,tree", [("5", "0"), ("5", "1"), ("4", "0"), ("4", "1"),
+                                          ("8", "-1")])
+def test_carries_under_injected_delays(cluster, tree):
     if not os.path.exists(DELAY_LIB):
         pytest.skip("libsat_delay.so not built")
-    env = dict(os.environ, SAT_LIBRARY=DELAY_LIB, SAT_CLUSTER=cluster)
+    env = dict(os.environ, SAT_LIBRARY=DELAY_LIB, SAT_CLUSTER=cluster, SAT_TREE=tree)
     out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], env=env, capture_output=True,
                          text=True, timeout=600)
     assert out.returncode == 0, out.stderr[-2000:]
     assert "BAD 0" in out.stdout, out.stdout[-2000:]
 
 
-@pytest.mark.parametrize("cluster", ["5", "4"])
-def test_lookback_ldg_variant_under_injected_delays(cluster):
-    """The same stress on the SAT_LB_LDG=1 build (look-back words read with
-    ld.relaxed.gpu -- the variant whose tag/value atomicity PTX guarantees)."""
+@pytest.mark.parametrize("cluster,tree", [("5", "0"), ("4", "0"), ("5", "1")])
+def test_carries_ldg_variant_under_injected_delays(cluster, tree):
+    """The same stress on the SAT_LB_LDG=1 build (look-back words and tree node
+    words read with ld.relaxed.gpu -- the variant whose per-word atomicity PTX
+    guarantees)."""
     if not os.path.exists(LDG_LIB):
         pytest.skip("libsat_delay_ldg.so not built")
-    env = dict(os.environ, SAT_LIBRARY=LDG_LIB, SAT_CLUSTER=cluster)
+    env = dict(os.environ, SAT_LIBRARY=LDG_LIB, SAT_CLUSTER=cluster, SAT_TREE=tree)
     out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], env=env, capture_output=True,
                          text=True, timeout=600)
     assert out.returncode == 0, out.stderr[-2000:]

@@ -2,7 +2,7 @@
 # Same-box A/B: tools/ab.sh SPEC [SPEC ...] -- times tools/quick.py (or $SCRIPT)
 # for each SPEC = <lib.so>[:VAR=VAL[,VAR=VAL...]] (env knobs of libsat),
 # interleaved twice so that pool-to-pool box variation cancels.
-for rep in 1 2; do
+for rep in $(seq 1 ${REPS:-2}); do
   for SPEC in "$@"; do
     L=${SPEC%%:*}
     ENVS=""
