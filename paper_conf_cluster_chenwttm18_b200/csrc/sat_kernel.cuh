@@ -585,7 +585,7 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) 
   }
 }
 #ifndef SAT_BO_CARRY
-#define SAT_BO_CARRY 0
+#define SAT_BO_CARRY 1
 #endif
 #ifndef SAT_BO_PROD
 #define SAT_BO_PROD 0
@@ -2402,11 +2402,11 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   }
 #endif
   SAT_PT(t0);
-#if SAT_BO_CARRY
-  mbar_wait_sleep(&sm.carry_full[t], (q / kNTot<P>) & 1);
-#else
-  mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
-#endif
+  // byte pairs: back-off polling (same-box A/B -0.4..-3%); floats: try_wait
+  if constexpr (SAT_BO_CARRY != 0 && (kBase<P> == P8U32S || kChan<P>))
+    mbar_wait_sleep(&sm.carry_full[t], (q / kNTot<P>) & 1);
+  else
+    mbar_wait(&sm.carry_full[t], (q / kNTot<P>) & 1);
   SAT_PT(t1);
   if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
   if (img >= 0) {
