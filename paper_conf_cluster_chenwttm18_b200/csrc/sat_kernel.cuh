@@ -698,6 +698,16 @@ __device__ __forceinline__ void mbar_arrive_remote(uint32_t rbar) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(rbar) : "memory");
 }
 
+// Waits for data that peers deliver into this CTA's shared memory with
+// st.async + complete_tx (aggregates, V_up): the phase cannot complete before
+// those bytes have landed here, so a CTA-scope acquire suffices for reading
+// them from shared memory; the cluster-scope form compiles to an L1
+// invalidation (CCTL.IVALL) per wait -- 5% of the 8u kernel's stall samples
+// (ncu r02b) on the carry path.  SAT_ACQ_CTA=0 restores the cluster scope.
+#ifndef SAT_ACQ_CTA
+#define SAT_ACQ_CTA 1
+#endif
+__device__ __forceinline__ void mbar_wait_peer_data(uint64_t* bar, uint32_t parity);
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
   uint32_t addr = smem_u32(bar);
   asm volatile(
@@ -707,6 +717,13 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
       "@!p bra WAITC_%=;\n\t}" ::"r"(addr),
       "r"(parity), "r"(0x100000u)
       : "memory");
+}
+__device__ __forceinline__ void mbar_wait_peer_data(uint64_t* bar, uint32_t parity) {
+#if SAT_ACQ_CTA
+  mbar_wait(bar, parity);
+#else
+  mbar_wait_cluster(bar, parity);
+#endif
 }
 
 __device__ __forceinline__ void cluster_sync_all() {
@@ -1953,7 +1970,7 @@ __device__ __forceinline__ void leader_warp(Smem<P, CL>& sm, const KParams& p, i
   for (uint32_t j = lw;; j += kNLW<P>) {
     const int ls = j % kNLead<P, CL>;
     SAT_PT(t0);
-    mbar_wait_cluster(&sm.lead_full[ls], (j / kNLead<P, CL>) & 1);
+    mbar_wait_peer_data(&sm.lead_full[ls], (j / kNLead<P, CL>) & 1);
     SAT_PT(t1);
     SAT_PADD(sm, kPfLbCluster, t1 - t0);
     const int64_t band = sm.lead_band[ls];
@@ -2595,7 +2612,7 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
       T = __shfl_sync(kFull, T, 0);
     }
     ++draws;
-    const bool done = T >= p.total_tickets;
+    const bool done = T < 0 || T >= p.total_tickets;  // T < 0: a counter out of step (never with plan-ordered launches)
     const int64_t g = T * CL + rank;
     const bool valid = !done && g < p.total_bands;
     const int64_t n = valid ? g / p.bands_per_image : 0;
@@ -2724,7 +2741,7 @@ __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
     for (uint32_t q = 0;; ++q) {
       mbar_wait(&sm.tot_full[q % kNTot<P>], (q / kNTot<P>) & 1);
       if (sm.tot_band[q % kNTot<P>] < 0) break;
-      mbar_wait_cluster(&sm.vin_full[q % kNV<P>], (q / kNV<P>) & 1);
+      mbar_wait_peer_data(&sm.vin_full[q % kNV<P>], (q / kNV<P>) & 1);
       offset_step<P, CL, kEx>(sm, p, q, lane);
     }
   } else if (warp >= kFirstLwWarp<P>) {

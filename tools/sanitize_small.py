@@ -1,6 +1,7 @@
 """Small SATs for compute-sanitizer runs (memcheck / synccheck / racecheck):
-every product kernel variant of round 2 on small shapes, results checked
-against the oracle (BAD 0 = all match)."""
+every product kernel variant of round 2 on small shapes -- cluster sizes 5 / 4
+/ 8, for 8u both carry mechanisms (look-back and the counted reduction tree)
+-- results checked against the oracle (BAD 0 = all match)."""
 import os
 import sys
 
@@ -22,19 +23,24 @@ def chk(ok, what):
         print("MISMATCH", what, flush=True)
 
 
+PAIR = {torch.uint8: sat.PAIR_8U_32S, torch.float32: sat.PAIR_32F_32F, torch.float64: sat.PAIR_64F_64F}
 for cl in ("5", "4", "8"):
-    os.environ["SAT_CLUSTER"] = cl
+    os.environ["SAT_CLUSTER"] = cl  # read at plan creation: one plan per cluster size
     for dt, H, W, N in [(torch.uint8, 300, 517, 1), (torch.float32, 200, 300, 1),
                         (torch.float64, 130, 129, 1), (torch.uint8, 70, 260, 3)]:
-        shape = (N, H, W) if N > 1 else (H, W)
-        x = torch.empty(shape, dtype=dt, device="cuda")
-        satgen.fill_device(x, seed=H)
-        y = sat.sat(x).cpu().numpy().reshape(N, H, W)
-        xs = x.cpu().numpy().reshape(N, H, W)
-        for n in range(N):
-            ref = oracle.sat(np.ascontiguousarray(xs[n]))
-            ok = np.array_equal(y[n], ref) if dt == torch.uint8 else np.allclose(y[n], ref, rtol=1e-4)
-            chk(ok, f"sat CL={cl} {dt} {shape}")
+        # integer pairs: both cross-cluster carry mechanisms (look-back, tree)
+        for mode in (("lookback", "tree") if dt == torch.uint8 else ("auto",)):
+            shape = (N, H, W) if N > 1 else (H, W)
+            plan = sat.Plan(PAIR[dt], H, W, N)
+            plan.set_carry(mode)
+            x = torch.empty(shape, dtype=dt, device="cuda")
+            satgen.fill_device(x, seed=H)
+            y = sat.sat(x, plan=plan).cpu().numpy().reshape(N, H, W)
+            xs = x.cpu().numpy().reshape(N, H, W)
+            for n in range(N):
+                ref = oracle.sat(np.ascontiguousarray(xs[n]))
+                ok = np.array_equal(y[n], ref) if dt == torch.uint8 else np.allclose(y[n], ref, rtol=1e-4)
+                chk(ok, f"sat CL={cl} {mode} {dt} {shape}")
 os.environ.pop("SAT_CLUSTER")
 # multi-channel pairs
 x = torch.empty((150, 333), dtype=torch.uint8, device="cuda")
