@@ -446,9 +446,6 @@ __device__ __forceinline__ uint64_t tl_now() {
   return t;
 }
 #endif
-#ifdef SAT_THROTTLE_NS
-__device__ unsigned int g_sat_smcnt[256];
-#endif
 enum ProfSlot {
   kPfComputeWaitFull = 0,   // warp 0: waiting for TMA data
   kPfComputeWaitCarry = 1,  // warp 0: waiting for the look-back result
@@ -513,7 +510,6 @@ struct __align__(128) Smem {
   int32_t tot_k[kNTot<P>];
   int32_t tot_chunk[kNTot<P>];
   volatile uint32_t passA_done;                 // chunks through pass A (ticket pacing)
-  uint32_t sm_slot;                             // experiment (SAT_THROTTLE_NS): arrival order on the SM
   uint8_t bin_of[256];                          // P8UHIST4: byte -> bin (from KParams, in smem:
                                                 // divergent constant-bank reads serialise)
 #ifdef SAT_PROFILE
@@ -2552,9 +2548,6 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
   }
 #else
   for (;;) {
-#ifdef SAT_THROTTLE_NS
-    if (!ended && sm.sm_slot == 0) __nanosleep(SAT_THROTTLE_NS);
-#endif
     if (!ended) {
       if (pass_a<P, CL>(sm, p, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
         ++qa;
@@ -2734,17 +2727,6 @@ __global__ void __launch_bounds__(kThreads<P>, kMinBlocks<P>)
     __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 
-#ifdef SAT_THROTTLE_NS
-  // Experiment: the first CTA to arrive on an SM (whose warps the scheduler
-  // favours) sleeps SAT_THROTTLE_NS before each pass A, to test whether evening
-  // out the two co-resident CTAs shortens the launch.
-  if (threadIdx.x == 0) {
-    uint32_t smid;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-    sm.sm_slot = atomicAdd(&g_sat_smcnt[smid & 255], 1u) & 1u;
-  }
-  __syncthreads();
-#endif
 #ifdef SAT_TIMELINE
   if (threadIdx.x == 0 && blockIdx.x < 1024) g_sat_tl[blockIdx.x][0] = tl_now();
 #endif
