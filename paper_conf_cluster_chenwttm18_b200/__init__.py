@@ -220,8 +220,8 @@ class Plan:
 _plans: dict = {}
 
 
-_KNOBS = ("SAT_FORCE_GENERIC", "SAT_CLUSTER", "SAT_SHORT", "SAT_MAX_CLUSTERS", "SAT_FORCE_CLUSTERS",
-          "SAT_LOG")
+_KNOBS = ("SAT_FORCE_GENERIC", "SAT_CLUSTER", "SAT_SHORT", "SAT_DEEP", "SAT_TREE", "SAT_MAX_CLUSTERS",
+          "SAT_FORCE_CLUSTERS", "SAT_LOG")
 
 
 def _plan_for(device, pair, h, w, batch) -> Plan:

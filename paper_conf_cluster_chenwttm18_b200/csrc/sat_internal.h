@@ -18,12 +18,14 @@ struct sat_plan_st {
   int num_sms = 0;
   int active_clusters[7][3][4] = {};  // [pair][cluster 2/4/8][mode: bit0 TMA, bit1 vec out]
   int active_short[7] = {};           // [pair] short-band variant, clusters of 4, TMA + vec out
+  int active_deep[7] = {};            // [pair] deep-ring variant (one CTA per SM), clusters of 4
   // Tuning / diagnosis knobs, read from the environment ONCE at plan creation
   // (SAT_FORCE_GENERIC, SAT_CLUSTER, SAT_SHORT, SAT_MAX_CLUSTERS,
   // SAT_FORCE_CLUSTERS, SAT_LOG); launches never consult the environment.
   int force_generic = 0;
   int cluster = 0;        // forced CTAs (bands) per cluster: 0 = by shape, else 2 / 4 / 8
   int short_bands = -1;   // -1 by shape, 0 / 1 forced
+  int deep_ring = -1;     // SAT_DEEP: -1 by shape, 0 / 1 forced
   int max_clusters = 0, force_clusters = 0;
   int log = 0;
   int tree_mode = -1;     // SAT_TREE: integer-pair carries -1 by shape, 0 look-back, 1 tree

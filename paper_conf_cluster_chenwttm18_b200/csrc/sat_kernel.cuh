@@ -162,7 +162,10 @@ struct Cfg<P64F64F> {
 #endif
   static constexpr int LOOK = SAT_LOOK64;
   static constexpr int NCW = 8;
-  static constexpr int NSTAGE = 3;
+#ifndef SAT_NST64
+#define SAT_NST64 4
+#endif
+  static constexpr int NSTAGE = SAT_NST64;
 };
 // 8u -> 32f (NPP's nppiIntegral_8u32f): the 8u->32s geometry (256-column
 // tiles, two 4-byte lane groups), fp32 values and scans.
@@ -277,6 +280,34 @@ template <>
 struct Cfg<P8U32F + kShort> : CfgShort<P8U32F> {};
 template <>
 struct Cfg<P32S32S + kShort> : CfgShort<P32S32S> {};
+
+// Deep-ring variants (P + kDeep): the pair's geometry with one CTA per SM, a
+// deeper TMA ring and twice the TMEM slots, for launches of at most one band
+// per SM (wide, short images: 4096 x 65536).  Two CTAs per SM would leave
+// half the slots empty there, and one CTA's bytes in flight (NSTAGE tiles)
+// bound its bandwidth: 64f 4096 x 65536 needs ~41 GB/s per band at 0.8 of
+// the copy peak against ~32 GB/s from three 16 KB stages.
+constexpr int kDeep = 16;
+template <int P>
+constexpr bool kIsShort = P >= kShort && P < kDeep;
+template <int P>
+constexpr bool kIsDeep = P >= kDeep;
+template <int P, int NST>
+struct CfgDeep : Cfg<P> {
+  static constexpr int MINB = 1;
+  static constexpr int NSTAGE = NST;
+  static constexpr int LOOK = 2 * Cfg<P>::LOOK + 1;  // 512 TMEM columns instead of 256
+};
+template <>
+struct Cfg<P8U32S + kDeep> : CfgDeep<P8U32S, 10> {};
+template <>
+struct Cfg<P32F32F + kDeep> : CfgDeep<P32F32F, 6> {};
+template <>
+struct Cfg<P64F64F + kDeep> : CfgDeep<P64F64F, 8> {};
+template <>
+struct Cfg<P8U32F + kDeep> : CfgDeep<P8U32F, 10> {};
+template <>
+struct Cfg<P32S32S + kDeep> : CfgDeep<P32S32S, 6> {};
 
 
 // Warp roles: NCW compute warps, the producer, the aggregate warp, the offset

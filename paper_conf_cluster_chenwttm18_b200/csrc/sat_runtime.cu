@@ -159,7 +159,7 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   int CL = default_cluster(kBase<P>, kp.total_bands);
   if (pl->cluster > 0) CL = pl->cluster;
   if (ex && CL != 4 && CL != 8) CL = 4;  // exclusive kernels: clusters of 4 and 8
-  if (P >= kShort) CL = 4;               // short-band kernels: clusters of 4 only
+  if (P >= kShort) CL = 4;               // short-band / deep-ring kernels: clusters of 4 only
   kp.total_tickets = (kp.total_bands + CL - 1) / CL;
   // Look-back workspace: one tagged carry vector per (cluster ticket, chunk).
   {
@@ -225,7 +225,9 @@ static sat_status launch_t(sat_plan_st* pl, const void* in, void* out, int64_t h
   const int ci = cluster_index(CL);
   // Persistent grid: every co-resident cluster slot, but no more clusters than tickets.
   int64_t clusters =
-      std::max(P >= kShort ? pl->active_short[kBase<P>] : pl->active_clusters[kBase<P>][ci][mode], 1);
+      std::max(kIsDeep<P> ? pl->active_deep[kBase<P>]
+               : P >= kShort ? pl->active_short[kBase<P>]
+                             : pl->active_clusters[kBase<P>][ci][mode], 1);
   if (pl->max_clusters > 0) clusters = std::min<int64_t>(clusters, pl->max_clusters);
   if (pl->force_clusters > 0) clusters = pl->force_clusters;
   clusters = std::min<int64_t>(clusters, kp.total_tickets);
@@ -417,6 +419,31 @@ static sat_status launch_dispatch(sat_plan_st* pl, const void* in, void* out, in
   const bool use_short = !ex && !multi_channel(pl->pair) && aligned && pl->force_generic == 0 &&
                          pl->cluster == 0 &&
                          (sh_env >= 0 ? sh_env == 1 : 2 * bands32 <= (int64_t)pl->num_sms);
+  // Deep-ring variant: at most one band per SM (and more than the short-band
+  // rule takes) -- one CTA per SM with a deeper TMA ring.  By shape for the
+  // 4-byte pairs only (4096 x 65536 32f -11%; 64f unchanged, 8u +4%, same-box
+  // A/B); SAT_DEEP=0/1 forces it for every pair.
+  const int dp_env = pl->deep_ring;
+  const bool deep_pair = pl->pair == SAT_32F_32F || pl->pair == SAT_32S_32S;
+  const bool use_deep = !use_short && !ex && !multi_channel(pl->pair) && aligned &&
+                        pl->force_generic == 0 && pl->cluster == 0 &&
+                        (dp_env >= 0 ? dp_env == 1 : deep_pair && bands32 <= (int64_t)pl->num_sms);
+  if (use_deep) {
+    switch (pl->pair) {
+      case SAT_8U_32S:
+        return launch_t<P8U32S + kDeep>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+      case SAT_32F_32F:
+        return launch_t<P32F32F + kDeep>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+      case SAT_64F_64F:
+        return launch_t<P64F64F + kDeep>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+      case SAT_8U_32F:
+        return launch_t<P8U32F + kDeep>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+      case SAT_32S_32S:
+        return launch_t<P32S32S + kDeep>(pl, in, out, h, w, ip, op, iis, ois, batch, carry_in, stream, ex, chain, hist);
+      default:
+        break;
+    }
+  }
   if (use_short) {
     switch (pl->pair) {
       case SAT_8U_32S:
@@ -546,12 +573,42 @@ static sat_status configure_short(sat_plan_st* pl) {
 }
 
 template <int P>
+static sat_status configure_deep(sat_plan_st* pl) {
+  constexpr int PD = P + kDeep, CL = 4;
+  const size_t smem = sizeof(Smem<PD, CL>);
+  cudaError_t e = cudaFuncSetAttribute(sat_occupancy_proxy<PD, CL>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sat_tile_kernel<PD, CL, true, true, false>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(deep)");
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(CL * 64);
+  cfg.blockDim = dim3(kThreads<PD>);
+  cfg.dynamicSmemBytes = smem;
+  cudaLaunchAttribute attr;
+  attr.id = cudaLaunchAttributeClusterDimension;
+  attr.val.clusterDim.x = CL;
+  attr.val.clusterDim.y = 1;
+  attr.val.clusterDim.z = 1;
+  cfg.attrs = &attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  e = cudaOccupancyMaxActiveClusters(&n, sat_occupancy_proxy<PD, CL>, &cfg);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters(deep)");
+  pl->active_deep[P] = std::min(n, pl->num_sms * (512 / kTmemCols<PD>) / CL);
+  return SAT_OK;
+}
+
+template <int P>
 static sat_status configure_t(sat_plan_st* pl) {
   sat_status st = configure_cl<P, SAT_CLX>(pl);
   if (st == SAT_OK) st = configure_cl<P, 4>(pl);
   if (st == SAT_OK) st = configure_cl<P, 8>(pl);
   if constexpr (!kChan<P>)
     if (st == SAT_OK) st = configure_short<P>(pl);
+  if constexpr (!kChan<P>)
+    if (st == SAT_OK) st = configure_deep<P>(pl);
   return st;
 }
 
@@ -701,6 +758,7 @@ sat_status sat_plan_create(sat_plan* plan, int device, sat_pair pair, int64_t ma
     pl->cluster = (c == SAT_CLX || c == 4 || c == 8) ? c : 0;
   }
   pl->short_bands = getenv_int("SAT_SHORT", -1);
+  pl->deep_ring = getenv_int("SAT_DEEP", -1);
   pl->max_clusters = getenv_int("SAT_MAX_CLUSTERS", 0);
   pl->force_clusters = getenv_int("SAT_FORCE_CLUSTERS", 0);
   pl->log = getenv_int("SAT_LOG", 0);
