@@ -975,47 +975,40 @@ __device__ __forceinline__ void rows_scan(const float* tile, int lane, float (&r
 template <int RW>
 __device__ __forceinline__ void rows_scan(const uint8_t* tile, int lane, float (&rowcarry)[RW],
                                           float (&R)[RW][2][4]) {
+  // The in-chunk prefixes of bytes are integers <= 65280: scan them exactly
+  // as the 8u->32s path does (dp4a group sums packed in 16-bit halves, one
+  // predicated-shuffle Kogge-Stone per row, dp4a in-group prefixes), then
+  // one rounding each: R = rowcarry + float(prefix), rowcarry += float(total).
   constexpr int TW = 256;
-  float p[RW][2][4], inc[RW][2];
-#pragma unroll
-  for (int i = 0; i < RW; ++i)
-#pragma unroll
-    for (int g = 0; g < 2; ++g) {
-      const uint32_t b = *reinterpret_cast<const uint32_t*>(tile + i * TW + g * 128 + 4 * lane);
-      p[i][g][0] = (float)(b & 0xffu);
-      p[i][g][1] = p[i][g][0] + (float)((b >> 8) & 0xffu);
-      p[i][g][2] = p[i][g][1] + (float)((b >> 16) & 0xffu);
-      p[i][g][3] = p[i][g][2] + (float)(b >> 24);
-      inc[i][g] = p[i][g][3];
-    }
-#pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    float o[RW][2];
-#pragma unroll
-    for (int i = 0; i < RW; ++i)
-#pragma unroll
-      for (int g = 0; g < 2; ++g) o[i][g] = __shfl_up_sync(kFull, inc[i][g], d);
-#pragma unroll
-    for (int i = 0; i < RW; ++i)
-#pragma unroll
-      for (int g = 0; g < 2; ++g)
-        if (lane >= d) inc[i][g] += o[i][g];
-  }
+  uint32_t w0[RW], w1[RW], own[RW], inc[RW];
 #pragma unroll
   for (int i = 0; i < RW; ++i) {
-    const float tot0 = __shfl_sync(kFull, inc[i][0], 31);
-    const float tot1 = __shfl_sync(kFull, inc[i][1], 31);
-    float ex0 = __shfl_up_sync(kFull, inc[i][0], 1);
-    float ex1 = __shfl_up_sync(kFull, inc[i][1], 1);
-    if (lane == 0) ex0 = ex1 = 0.0f;
-    const float base0 = rowcarry[i] + ex0;
-    const float base1 = (rowcarry[i] + tot0) + ex1;
-    rowcarry[i] = (rowcarry[i] + tot0) + tot1;
+    w0[i] = *reinterpret_cast<const uint32_t*>(tile + i * TW + 4 * lane);
+    w1[i] = *reinterpret_cast<const uint32_t*>(tile + i * TW + 128 + 4 * lane);
+    own[i] = __dp4a(w0[i], 0x01010101u, 0u) | (__dp4a(w1[i], 0x01010101u, 0u) << 16);
+    inc[i] = own[i];
+  }
 #pragma unroll
-    for (int e = 0; e < 4; ++e) {
-      R[i][0][e] = base0 + p[i][0][e];
-      R[i][1][e] = base1 + p[i][1][e];
-    }
+  for (int d = 1; d < 32; d <<= 1)  // Alg. 3, lane >= d (reading R10)
+#pragma unroll
+    for (int i = 0; i < RW; ++i) ks_step(inc[i], d);
+#pragma unroll
+  for (int i = 0; i < RW; ++i) {
+    const uint32_t tot = __shfl_sync(kFull, inc[i], 31);
+    const uint32_t ex = inc[i] - own[i];
+    const uint32_t tot0 = tot & 0xFFFFu;
+    const uint32_t base0 = ex & 0xFFFFu;
+    const uint32_t base1 = tot0 + (ex >> 16);
+    const float rc = rowcarry[i];
+    rowcarry[i] = rc + (float)(tot0 + (tot >> 16));
+    R[i][0][0] = rc + (float)__dp4a(w0[i], 0x00000001u, base0);
+    R[i][0][1] = rc + (float)__dp4a(w0[i], 0x00000101u, base0);
+    R[i][0][2] = rc + (float)__dp4a(w0[i], 0x00010101u, base0);
+    R[i][0][3] = rc + (float)__dp4a(w0[i], 0x01010101u, base0);
+    R[i][1][0] = rc + (float)__dp4a(w1[i], 0x00000001u, base1);
+    R[i][1][1] = rc + (float)__dp4a(w1[i], 0x00000101u, base1);
+    R[i][1][2] = rc + (float)__dp4a(w1[i], 0x00010101u, base1);
+    R[i][1][3] = rc + (float)__dp4a(w1[i], 0x01010101u, base1);
   }
 }
 
