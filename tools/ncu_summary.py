@@ -46,6 +46,8 @@ WORKLOAD_OF = {  # prof_one args -> bench workload name
     "p6_16384x16384x1": "hist4-16384sq-8u",
     "p1_8192x8192x1": "sweep-8192sq-32f32f",
     "p2_4096x65536x1": "64f-4096x65536",
+    "p3_16384x16384x1": "8u32f-16384sq",
+    "p1_4096x65536x1": "32f-4096x65536",
 }
 IN_B = {0: 1, 1: 4, 2: 8, 3: 1, 4: 4, 5: 1, 6: 1}
 OUT_B = {0: 4, 1: 4, 2: 8, 3: 4, 4: 4, 5: 8, 6: 16}
