@@ -1191,27 +1191,25 @@ __device__ __forceinline__ void rows_scan_xf(const uint8_t* tile, int lane, cons
       }
       inc[i][g] = R[i][g][C::E - 1];
     }
+  // a3 per channel with predicated-shuffle steps; the exclusive prefix is
+  // inc - own (wrap-around u32, exact) instead of a further shuffle
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    TB o[RW][C::G];
-#pragma unroll
-    for (int i = 0; i < RW; ++i)
-#pragma unroll
-      for (int g = 0; g < C::G; ++g) o[i][g] = shfl_up(inc[i][g], d);
+  for (int d = 1; d < 32; d <<= 1)
 #pragma unroll
     for (int i = 0; i < RW; ++i)
 #pragma unroll
       for (int g = 0; g < C::G; ++g)
-        if (lane >= d) inc[i][g] += o[i][g];
-  }
+#pragma unroll
+        for (int k = 0; k < C::K; ++k) ks_step(inc[i][g].c[k], d);
 #pragma unroll
   for (int i = 0; i < RW; ++i) {
     TB base = rowcarry[i];
 #pragma unroll
     for (int g = 0; g < C::G; ++g) {
       const TB tot = shfl_idx(inc[i][g], 31);
-      TB ex = shfl_up(inc[i][g], 1);
-      if (lane == 0) ex = TB(0);
+      TB ex;
+#pragma unroll
+      for (int k = 0; k < C::K; ++k) ex.c[k] = inc[i][g].c[k] - R[i][g][C::E - 1].c[k];
       const TB bx = base + ex;
 #pragma unroll
       for (int e = 0; e < C::E; ++e) R[i][g][e] = bx + R[i][g][e];
