@@ -1134,18 +1134,11 @@ __device__ __forceinline__ void rows_scan_hist4(const uint8_t* tile, int lane, c
 #pragma unroll
     for (int g = 0; g < 2; ++g) inc[i][g] = own[i][g] = hist_pack(tile[i * TW + g * 32 + lane], lut, bin0);
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    uint32_t o[RW][2];
+  for (int d = 1; d < 32; d <<= 1)
 #pragma unroll
     for (int i = 0; i < RW; ++i)
 #pragma unroll
-      for (int g = 0; g < 2; ++g) o[i][g] = __shfl_up_sync(kFull, inc[i][g], d);
-#pragma unroll
-    for (int i = 0; i < RW; ++i)
-#pragma unroll
-      for (int g = 0; g < 2; ++g)
-        if (lane >= d) inc[i][g] += o[i][g];
-  }
+      for (int g = 0; g < 2; ++g) ks_step(inc[i][g], d);
 #pragma unroll
   for (int i = 0; i < RW; ++i) {
     const uint32_t t0 = __shfl_sync(kFull, inc[i][0], 31), t1 = __shfl_sync(kFull, inc[i][1], 31);
