@@ -618,9 +618,6 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) 
 #ifndef SAT_BO_CARRY
 #define SAT_BO_CARRY 1
 #endif
-#ifndef SAT_BO_PROD
-#define SAT_BO_PROD 0
-#endif
 
 __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, uint64_t* bar,
                                             int32_t x, int32_t y, int32_t z, uint64_t policy) {
@@ -824,11 +821,6 @@ __device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&v)[16]) {
       : "r"(taddr)
       : "memory");
 }
-// SAT_DEFER_ST=1: pass A does not wait for its TMEM stores; pass B waits
-// (tcgen05.wait::st) just before it loads a slot back.
-#ifndef SAT_DEFER_ST
-#define SAT_DEFER_ST 0
-#endif
 __device__ __forceinline__ void tmem_wait_st() {
   asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }
@@ -2349,9 +2341,7 @@ __device__ __forceinline__ bool pass_a(Smem<P, CL>& sm, const KParams& p, uint32
         put_words<TB>(w, (i * C::G + g) * C::E + e, acc[g][e]);
       }
   tmem_st(tmem_addr(sm, t, warp), w);
-#if !SAT_DEFER_ST
   tmem_wait_st();
-#endif
   // a4: this warp's column totals for the block partial-sum scan.
 #pragma unroll
   for (int g = 0; g < C::G; ++g)
@@ -2427,13 +2417,6 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   const int t = q % kNTot<P>;
   const int32_t img = sm.meta[warp][t][1];  // written by this warp's pass A
   uint32_t w[NW];
-#if SAT_DEFER_ST
-  // S' back from TMEM first: the load's latency overlaps the carry wait
-  if (img >= 0) {
-    tmem_wait_st();  // pass A's stores (the latest one an iteration ago) have landed
-    tmem_ld(tmem_addr(sm, t, warp), w);
-  }
-#endif
   SAT_PT(t0);
   // byte pairs: back-off polling (same-box A/B -0.4..-3%); floats: try_wait
   if constexpr (SAT_BO_CARRY != 0 && (kBase<P> == P8U32S || kChan<P>))
@@ -2443,9 +2426,7 @@ __device__ __forceinline__ void pass_b(Smem<P, CL>& sm, const KParams& p, uint32
   SAT_PT(t1);
   if (warp == 0) SAT_PADD(sm, kPfComputeWaitCarry, t1 - t0);
   if (img >= 0) {
-#if !SAT_DEFER_ST
     tmem_ld(tmem_addr(sm, t, warp), w);
-#endif
     TB off[C::G][C::E];  // V_up + the warps above + nVal (offset warp)
 #pragma unroll
     for (int g = 0; g < C::G; ++g)
@@ -2542,26 +2523,6 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
   for (int i = 0; i < RW; ++i) rowcarry[i] = TB(0);
   uint32_t qa = 0, qb = 0;
   bool ended = false;
-  // Pass B of chunk q runs right after pass A of chunk q + LOOK, at the top of
-  // the next iteration (so pass A's TMEM stores have an iteration to land
-  // before a TMEM load waits for them); before pass A(qa), qa - qb <= LOOK,
-  // i.e. the slot qa reuses (qa - LOOK - 1) has been drained.
-#if SAT_DEFER_ST
-  for (;;) {
-    if (qb < qa && (ended || qa - qb > (uint32_t)C::LOOK)) {
-      pass_b<P, CL, kVecOut, kEx>(sm, p, qb, warp, lane, prevlast);
-      ++qb;
-    }
-    if (!ended) {
-      if (pass_a<P, CL>(sm, p, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
-        ++qa;
-      else
-        ended = true;
-    } else if (qb == qa) {
-      break;
-    }
-  }
-#else
   for (;;) {
     if (!ended) {
       if (pass_a<P, CL>(sm, p, qa, qa % C::NSTAGE, (qa / C::NSTAGE) & 1, rowcarry, warp, lane))
@@ -2576,7 +2537,6 @@ __device__ __forceinline__ void compute_warp(Smem<P, CL>& sm, const KParams& p, 
       break;
     }
   }
-#endif
   // End-of-work sentinel for the offset warp (the slot is free: all pass B done).
   {
     const int t = qa % kNTot<P>;
@@ -2636,11 +2596,7 @@ __device__ __forceinline__ void producer_warp(Smem<P, CL>& sm, const KParams& p,
     const int32_t nch = done ? 1 : p.nchunks;
     for (int32_t c = 0; c < nch; ++c, ++q) {
       const int s = q % C::NSTAGE;
-#if SAT_BO_PROD
-      mbar_wait_sleep(&sm.empty[s], ((q / C::NSTAGE) & 1) ^ 1u);
-#else
       mbar_wait(&sm.empty[s], ((q / C::NSTAGE) & 1) ^ 1u);
-#endif
       if (done) {
         if (lane == 0) {
           sm.stage_band[s] = -1;
