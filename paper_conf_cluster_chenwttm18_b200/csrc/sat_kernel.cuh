@@ -637,8 +637,11 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
 
 
 // Streaming (evict-first) 16-byte output store.
+#ifndef SAT_ST_HINT
+#define SAT_ST_HINT ".cs"
+#endif
 __device__ __forceinline__ void st_cs_v4(void* p, uint4 v) {
-  asm volatile("st.global.cs.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y),
+  asm volatile("st.global" SAT_ST_HINT ".v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y),
                "r"(v.z), "r"(v.w)
                : "memory");
 }
